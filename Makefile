@@ -1,0 +1,37 @@
+# Builds the three native libraries in-tree (the .so files travel to the GPU
+# box with the gpurun snapshot; they are git-ignored).
+#   paper_conf_isca_shaharbs16_b200/libapointer.so  -- the product (CUDA, sm_100a)
+#   oracle/liboracle.so                             -- CPU oracle (test infrastructure)
+#   synth/libsynth.so                               -- seeded input generators
+NVCC    ?= /usr/local/cuda/bin/nvcc
+HOSTCC  := $(shell test -x /usr/bin/gcc && echo /usr/bin/gcc || echo gcc)
+PKG     := paper_conf_isca_shaharbs16_b200
+CSRC    := $(PKG)/csrc
+ARCH    := -gencode arch=compute_100a,code=sm_100a
+NVFLAGS := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -Wall \
+           -Iinclude -I$(CSRC) --expt-relaxed-constexpr
+CFLAGS  := -O2 -fopenmp -fPIC -Wall -Wextra -std=c11
+
+CU_SRCS := $(wildcard $(CSRC)/*.cu)
+CU_HDRS := $(wildcard $(CSRC)/*.cuh) $(wildcard include/*.h) $(wildcard include/ap/*.cuh)
+
+all: synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so
+
+synth/libsynth.so: synth/synth.c
+	$(HOSTCC) $(CFLAGS) -shared $< -o $@
+
+oracle/liboracle.so: oracle/oracle.c
+	$(HOSTCC) $(CFLAGS) -shared $< -o $@
+
+$(PKG)/libapointer.so: $(CU_SRCS) $(CU_HDRS)
+	$(NVCC) $(NVFLAGS) -shared $(CU_SRCS) -o $@ -lcuda
+
+host: synth/libsynth.so oracle/liboracle.so
+
+sass: $(PKG)/libapointer.so
+	/usr/local/cuda/bin/cuobjdump -sass $< > build_sass.txt
+
+clean:
+	rm -f synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so
+
+.PHONY: all host clean sass
