@@ -1,0 +1,233 @@
+/*
+ * ap.h — C ABI of the B200 apointer library (libapointer.so).
+ *
+ * ActivePointers (Shahar, Bergman, Silberstein, ISCA'16): a file mapped into
+ * GPU memory is read through "active pointers" that translate file offsets in
+ * software, cache the translation in a register, and take page faults that
+ * are handled on the GPU (PAPER.md:9-13 abstract; §III, §IV).  This header is
+ * the host-side boundary: create a page cache in HBM, map a "file" that lives
+ * in pinned host memory, run the paper's microbenchmarks and its photo
+ * collage, read statistics.  The device-side pointer type is in
+ * include/ap/apointer.cuh.
+ *
+ * Conventions (every function):
+ *   - returns int: AP_OK (0) on success, a negative AP_E* code on failure;
+ *   - never throws, never aborts, writes results through out-parameters only
+ *     on success;
+ *   - pointers named *_dev are device pointers (cudaMalloc / torch CUDA
+ *     tensors) owned by the caller; *_host are ordinary host pointers owned by
+ *     the caller; the library never frees caller memory;
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream); asynchronous calls enqueue on it and return immediately;
+ *   - a cache is bound to one device; calls switch to that device and
+ *     restore the caller's current device before returning;
+ *   - calls on one cache are not thread-safe against each other.
+ */
+#ifndef AP_H_
+#define AP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---------------------------------------------------------------- errors */
+#define AP_OK 0
+#define AP_EINVAL (-1)    /* bad argument                                   */
+#define AP_ENOMEM (-2)    /* device or pinned-host allocation failed         */
+#define AP_ECUDA (-3)     /* a CUDA runtime call failed                      */
+#define AP_EBUSY (-4)     /* live references / mapped regions prevent it     */
+#define AP_ERANGE (-5)    /* region id / size / offset outside the layout    */
+#define AP_EFAULT (-6)    /* device: dereference past the region or misaligned */
+#define AP_ENOFRAME (-7)  /* device: no evictable frame (all pinned)         */
+#define AP_ETIMEDOUT (-8) /* device: fault-path watchdog expired             */
+
+/* Human-readable text for an AP_* code (static storage, never NULL). */
+const char* ap_strerror(int code);
+
+/* ------------------------------------------------------------- the cache */
+typedef struct ap_cache_s* ap_cache_t;
+typedef uint32_t ap_region_t;
+
+/* ap_cache_create — the GPU page cache (§V "page cache in
+ * GPU memory"; frames of page_size bytes, PAPER.md:363 uses 4 KB).
+ *   frames     number of page frames, 1 <= frames < 2^29
+ *   page_size  bytes per page: a power of two in [4096, 2 MiB]
+ *   device     CUDA device ordinal
+ * Allocates frames*page_size bytes of HBM (page_size aligned), the frame
+ * owner table (8 B/frame), the free-frame array (4 B/frame), statistics and
+ * the region table.  Errors: AP_EINVAL (bad size), AP_ENOMEM (HBM),
+ * AP_ECUDA. */
+int ap_cache_create(uint64_t frames, uint32_t page_size, int device, ap_cache_t* out);
+
+/* Frees everything. AP_EBUSY while regions are still mapped. */
+int ap_cache_destroy(ap_cache_t cache);
+
+/* ap_mmap — map a read-only "file" (PAPER.md:125, 131 gvmmap(size, O_RDONLY,
+ * fd, foffset); the file lives in host RAM as in PAPER.md:367, 428).
+ *   host_buf  the file bytes in host memory, 16-B aligned, caller-owned; it
+ *             must stay valid and unmodified until ap_munmap.  If it is not
+ *             already page-locked it is registered (cudaHostRegisterMapped |
+ *             ReadOnly) here and unregistered by ap_munmap.
+ *   bytes     file size, > 0 (a ragged last page is zero-padded in its frame)
+ * Creates the region's page table: one 8-B PTE per page, all EMPTY.
+ * Errors: AP_EINVAL (NULL, 0 bytes, misaligned), AP_ERANGE (65535 regions
+ * mapped, or > 2^48 pages), AP_ENOMEM, AP_ECUDA. */
+int ap_mmap(ap_cache_t cache, const void* host_buf, uint64_t bytes, ap_region_t* out);
+
+/* Unmap: frames holding the region's pages go back to the free list.
+ * AP_EBUSY if any page of the region still has a positive reference count
+ * (a linked apointer). */
+int ap_munmap(ap_cache_t cache, ap_region_t region);
+
+/* Device-accessible alias of the region's host bytes (the zero-copy view the
+ * fault path fills from). Useful for raw-pointer twins. */
+int ap_region_devptr(ap_cache_t cache, ap_region_t region, const void** out);
+
+/* ------------------------------------------------------------ statistics */
+typedef struct {
+    uint64_t major;       /* major faults = page fills            */
+    uint64_t minor;       /* minor faults = links to a resident page              */
+    uint64_t fill_bytes;  /* bytes read from host memory by fills                 */
+    uint64_t evictions;   /* frames reclaimed from refcount-0 pages               */
+    uint64_t waits;       /* fault rounds that had to back off                    */
+    uint64_t downgrades;  /* lanes proactively unlinked under frame pressure      */
+    uint64_t nofree;      /* allocation attempts that found no evictable frame    */
+    uint64_t unlinks;     /* warp-aggregated reference-count decrements           */
+} ap_stats_t;
+
+/* Sum of the device counters since create/reset (synchronises the device). */
+int ap_cache_stats(ap_cache_t cache, ap_stats_t* out);
+
+/* Evict every page, rebuild the free list, zero the counters: the next run
+ * starts cold ("clearing the GPU buffer cache between runs").
+ * AP_EBUSY if any page has a positive reference count. Synchronises. */
+int ap_cache_reset(ap_cache_t cache);
+
+/* Victim-selection policy of the eviction path.
+ *   AP_POLICY_CLOCK   second-chance clock over frames (default)
+ *   AP_POLICY_RANDOM  random victims from `seed` (test-only: output must not
+ *                     depend on eviction order)                         */
+#define AP_POLICY_CLOCK 0
+#define AP_POLICY_RANDOM 1
+int ap_cache_set_policy(ap_cache_t cache, int policy, uint64_t seed);
+
+/* Fault-path tunables: max_claims = pages one warp claims per fault round
+ * (1 = the paper's sequential handling); sweep_steps = clock
+ * steps (32 frames each) before an allocation gives up and backs off;
+ * timeout_ms = watchdog for one dereference (0 = default 20000). */
+int ap_cache_set_tuning(ap_cache_t cache, uint32_t max_claims, uint32_t sweep_steps,
+                        uint32_t timeout_ms);
+
+/* Sticky device error word (AP_EFAULT / AP_ENOFRAME / AP_ETIMEDOUT), cleared
+ * on read; AP_OK if none. Synchronises. */
+int ap_last_device_error(ap_cache_t cache);
+
+/* Debug dumps for the invariant checks (synchronise):
+ *   owner_host[frames]  0 = none, else ((region+1) << 48) | page
+ *   free_left           frames still on the free list
+ *   pte_host[npages]    bits 63:62 state (0 EMPTY, 1 LOADING, 2 VALID),
+ *                       61 reference bit, 60:32 frame, 31:0 reference count */
+int ap_cache_dump(ap_cache_t cache, uint64_t* owner_host, uint64_t* free_left);
+int ap_region_npages(ap_cache_t cache, ap_region_t region, uint64_t* npages);
+int ap_region_dump_pte(ap_cache_t cache, ap_region_t region, uint64_t* pte_host);
+
+/* Fault pages [first_page, first_page+npages) of a region into the cache
+ * (one warp per page dereferences it through an apointer); they stay
+ * resident with reference count 0. Asynchronous on `stream`. */
+int ap_prefill(ap_cache_t cache, ap_region_t region, uint64_t first_page, uint64_t npages,
+               void* stream);
+
+/* ------------------------------------------------- microbenchmark (§VI-A/C) */
+#define AP_SEQ 0       /* warp w reads units w, w+W, ... sequentially         */
+#define AP_UNIFORM 1   /* uniform-random element offsets                      */
+#define AP_DIVERGENT 2 /* the 32 lanes of a warp on 32 distinct pages         */
+
+#define AP_MODE_APOINTER 0 /* read through ap::ptr<T> (the method)           */
+#define AP_MODE_RAW 1      /* identical kernel on a raw pointer (the twin,     *
+                            * PAPER.md:304 "two versions of every benchmark") */
+
+typedef struct {
+    int32_t pattern;           /* AP_SEQ | AP_UNIFORM | AP_DIVERGENT             */
+    uint32_t elem_bytes;       /* 4, 8 or 16                                     */
+    uint32_t grid, block;      /* launch shape; block a multiple of 32, <= 1024  */
+    uint32_t reads_per_thread; /* UNIFORM / DIVERGENT                            */
+    uint32_t passes;           /* SEQ: sweeps over [0, span)                     */
+    uint32_t unit_bytes;       /* SEQ: bytes per warp unit (multiple of 32*elem, *
+                                *      divides the page size)                    */
+    uint32_t page_bytes;       /* DIVERGENT: page size of the pattern            */
+    uint64_t span_bytes;       /* SEQ: bytes swept (0 = whole region)            */
+    uint64_t seed;             /* UNIFORM / DIVERGENT offset generator seed       */
+    int32_t mode;              /* AP_MODE_APOINTER | AP_MODE_RAW                 */
+    int32_t out_copy;          /* SEQ: out receives the bytes read at their      *
+                                * offsets (span bytes) instead of checksums      */
+    const void* raw_base;      /* AP_MODE_RAW: device-readable file bytes (an HBM *
+                                * copy, or ap_region_devptr for zero-copy)       */
+} ap_bench_cfg;
+
+/* Run one microbenchmark launch (asynchronous on `stream`).
+ * out_dev: uint64[grid*block] per-thread FNV-1a-64 checksums over the values
+ * the thread read in access order, or
+ * span bytes when out_copy.  Errors: AP_EINVAL (cfg), AP_ECUDA (launch). */
+int ap_bench_read(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg, void* out_dev,
+                  void* stream);
+
+/* End-to-end variant: the same launch with the result copied into host
+ * memory (out_host, caller-owned), synchronising; *seconds = wall time of
+ * launch + device->host copy measured with CUDA events. */
+int ap_bench_read_host(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg,
+                       void* out_host, double* seconds);
+
+/* ---------------------------------------------------- photo collage (§VI-E) */
+typedef struct {
+    const uint8_t* target_dev;   /* W*H*3 uint8 RGB, interleaved, row-major       */
+    uint32_t W, H;               /* multiples of 32                               */
+    uint32_t L, K;               /* LSH tables, projections per table (K <= 16)   */
+    uint32_t bucket_bits;        /* 1..30: buckets per table = 2^bucket_bits       */
+    int32_t w;                   /* LSH bucket width, > 0                          */
+    const int16_t* proj_dev;     /* [L][K][768]                                    */
+    const int32_t* bias_dev;     /* [L][K]                                         */
+    const uint32_t* offsets_dev; /* [L][2^bucket_bits + 1] bucket CSR offsets      */
+    const uint32_t* ids_dev;     /* [L][N] record ids, ascending per bucket        */
+    uint64_t N;                  /* records in the file                            */
+    uint32_t rec_stride;         /* bytes between records (4096 = padded, 3072)   */
+    uint32_t group;              /* candidates per warp iteration: 1, 2 or 4       */
+    uint64_t block_begin;        /* first query block (row-major 32x32 blocks)     */
+    uint64_t block_count;        /* number of query blocks                        */
+    int32_t mode;                /* AP_MODE_APOINTER | AP_MODE_RAW                 */
+    const void* raw_base;        /* AP_MODE_RAW: device-readable record file       */
+} ap_collage_in;
+
+/* ap_collage_run — the collage kernel ("calculates the
+ * histogram of each 32x32 block, computes its LSH keys, reads the candidate
+ * histograms from the respective buckets stored in a file, exhaustively
+ * searches for the closest ones among the candidates, and in the end produces
+ * the indexes of the images"; all in one kernel).  Records are read through
+ * apointers over `records` (mode APOINTER).  winners_dev: uint32
+ * [block_count][2] = (image index, squared Euclidean distance); a block with
+ * no candidate gets (0xFFFFFFFF, 0xFFFFFFFF).  Asynchronous on `stream`.
+ * Errors: AP_EINVAL (W/H not multiples of 32, K > 16, group), AP_ECUDA. */
+int ap_collage_run(ap_cache_t cache, ap_region_t records, const ap_collage_in* in,
+                   uint32_t* winners_dev, void* stream);
+
+/* ap_lsh_build_index — the dataset index ("The dataset images
+ * are placed in buckets indexed by the LSH keys derived from their
+ * histograms").  Reads the N records of `records` (zero-copy from host
+ * memory), computes each record's L keys, and writes per table the bucket
+ * CSR: offsets_dev [L][2^bucket_bits+1], ids_dev [L][N] (ascending within a
+ * bucket).  Synchronises `stream` before returning (it allocates scratch).
+ * Errors: AP_EINVAL, AP_ENOMEM, AP_ECUDA. */
+int ap_lsh_build_index(ap_cache_t cache, ap_region_t records, uint64_t N, uint32_t rec_stride,
+                       uint32_t L, uint32_t K, uint32_t bucket_bits, int32_t w,
+                       const int16_t* proj_dev, const int32_t* bias_dev, uint32_t* offsets_dev,
+                       uint32_t* ids_dev, void* stream);
+
+/* -------------------------------------------------------------- utilities */
+/* Library version string and the compile target (static storage). */
+const char* ap_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* AP_H_ */

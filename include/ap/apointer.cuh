@@ -1,0 +1,630 @@
+/*
+ * ap/apointer.cuh — the device side of ActivePointers on B200 (sm_100a).
+ *
+ * An apointer (§III-C, Fig. 3) is a pointer into a file
+ * mapped with ap_mmap.  It is read like a normal pointer; under the hood:
+ *
+ *   translation field (Fig. 5; long apointer, R-A16):
+ *     one 64-bit register, bit 63 = valid ("linked"), bits 62:61 permission
+ *     (reserved; checks are off as in PAPER.md:308), bits 60:0 = the device
+ *     address of the datum in the HBM page cache when linked (the "aphysical"
+ *     address), or the region-relative file offset (the "xAddress") when
+ *     unlinked.  A linked dereference is `and` + `ld`: no lookup, the
+ *     register is the TLB.
+ *   metadata: region descriptor pointer, linked page number,
+ *     log2(page size); only the fault path and page-crossing arithmetic read it.
+ *
+ * Hit path: the data load is issued speculatively
+ * from the masked address while the warp votes on the valid bit; if every
+ * active lane is linked the loaded value is returned.  Unlinked lanes load
+ * from the region descriptor instead (always mapped; R-A21), the value is
+ * discarded.
+ *
+ * Fault path (§III-D, Listing 1; cleaned
+ * reading R-A9): translation aggregation.  Lanes on the same page form a
+ * group with __match_any_sync; the lowest lane is its leader and the only
+ * lane touching shared structures; the reference count grows by popc(group).
+ * Minor faults (page resident) are lock-free CASes on the page-table entry
+ * and may proceed for all groups at once (R-A13).  Major faults claim the
+ * entry (EMPTY -> LOADING), take a frame from the free list or by clock
+ * eviction of a refcount-0 page, and the whole warp copies the
+ * page from pinned host memory over the host link with 16-B loads; then a
+ * release store publishes VALID (R-A15).  Distinct major faults of a warp are
+ * handled one page per round by default.
+ *
+ * Reference counts (Fig. 4): +popc on link;
+ * -popc (warp aggregated, release) when a pointer leaves its page, is
+ * assigned, copied from, or destroyed; under frame pressure a warp also
+ * proactively unlinks lanes it already served in the current dereference
+ * (the "heuristic" of PAPER.md:115, R-A19/A20).
+ *
+ * Usage rules: the lanes of a warp that call an operation together must be
+ * converged (the operation uses __activemask()); all lanes of one call use
+ * pointers into the same cache; sizeof(T) is 4, 8 or 16 and offsets are
+ * multiples of sizeof(T) (a T never straddles a page).
+ */
+#ifndef AP_APOINTER_CUH_
+#define AP_APOINTER_CUH_
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+/* The fault path is kept out of line by default so the hit path stays a
+ * handful of instructions; -DAP_SLOW_INLINE inlines it. */
+#ifndef AP_SLOW_ATTR
+#ifdef AP_SLOW_INLINE
+#define AP_SLOW_ATTR __forceinline__
+#else
+#define AP_SLOW_ATTR __noinline__
+#endif
+#endif
+
+namespace ap {
+
+/* ------------------------------------------------------------ layouts */
+/* Page-table entry (R-A17): [63:62] state, [61] reference bit,
+ * [60:32] frame, [31:0] reference count. */
+constexpr uint64_t PTE_EMPTY = 0ull;
+constexpr uint64_t PTE_LOADING = 1ull << 62;
+constexpr uint64_t PTE_VALID = 2ull << 62;
+constexpr uint64_t PTE_REF = 1ull << 61;
+constexpr uint64_t PTE_FRAME_MASK = (1ull << 29) - 1;
+constexpr uint64_t PTE_RC_MASK = 0xffffffffull;
+
+/* Translation field (R-A16). */
+constexpr uint64_t XL_VALID = 1ull << 63;
+constexpr uint64_t XL_ADDR = (1ull << 61) - 1;
+
+constexpr uint64_t PAGE_MASK48 = (1ull << 48) - 1;
+
+/* Device error codes (mirror include/ap.h). */
+constexpr int ERR_FAULT = -6;
+constexpr int ERR_NOFRAME = -7;
+constexpr int ERR_TIMEDOUT = -8;
+
+constexpr int POLICY_CLOCK = 0;
+constexpr int POLICY_RANDOM = 1;
+
+/* Counters, sharded by SM to keep atomics off one address. */
+struct alignas(64) dev_stats {
+    unsigned long long major, minor, fill_bytes, evictions, waits, downgrades, nofree, unlinks;
+};
+constexpr int STAT_SHARDS = 64;
+
+struct dev_cache;
+
+/* Region descriptor (one mapped file), 64-B aligned in device memory. */
+struct alignas(64) dev_region {
+    const uint8_t* host;    /* device alias of the pinned host bytes      */
+    uint64_t bytes;         /* file size                                  */
+    uint64_t npages;        /* ceil(bytes / page)                         */
+    uint64_t* pte;          /* npages entries                             */
+    const dev_cache* cache; /* owning cache                               */
+    uint32_t id;            /* region id (< 65535)                        */
+    uint32_t live;          /* 1 while mapped                             */
+    uint64_t pad_[2];
+};
+
+/* Cache descriptor, one copy in device memory per ap_cache_t. */
+struct alignas(64) dev_cache {
+    uint8_t* pool;                  /* frames * page bytes, page aligned   */
+    uint64_t* owner;                /* [frames] ((region+1)<<48)|page, 0   */
+    const uint32_t* free_ids;       /* [nfree] free frame ids              */
+    unsigned long long* free_head;  /* pop counter                         */
+    unsigned long long* clock_hand; /* clock position (frames, mod)        */
+    dev_region* regions;            /* region table                        */
+    dev_stats* stats;               /* [STAT_SHARDS]                       */
+    int* err;                       /* sticky error word                   */
+    uint64_t frames;
+    uint64_t nfree;
+    uint64_t policy_seed;
+    uint64_t timeout_ns;
+    uint32_t log2_page;
+    int32_t policy;
+    uint32_t max_claims;
+    uint32_t sweep_steps;
+};
+
+/* ---------------------------------------------------- PTX helpers (A15) */
+namespace detail {
+
+__device__ __forceinline__ unsigned lane_id() {
+    unsigned l;
+    asm volatile("mov.u32 %0, %%laneid;" : "=r"(l));
+    return l;
+}
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+__device__ __forceinline__ unsigned sm_id() {
+    unsigned s;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+    return s;
+}
+__device__ __forceinline__ uint64_t now_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t cas_acq_rel(uint64_t* p, uint64_t cmp, uint64_t val) {
+    uint64_t old;
+    asm volatile("atom.acq_rel.gpu.global.cas.b64 %0, [%1], %2, %3;"
+                 : "=l"(old) : "l"(p), "l"(cmp), "l"(val) : "memory");
+    return old;
+}
+__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) {
+    asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+__device__ __forceinline__ uint64_t sm64(uint64_t x) {
+    uint64_t z = x + 0x9e3779b97f4a7c15ull;
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+    return z ^ (z >> 31);
+}
+
+/* Frame-data loads bypass L1 (.cg): a recycled frame can never be served
+ * from a stale L1 line, and the data is streamed once anyway. */
+template <class T> __device__ __forceinline__ T ld_data(const T* p);
+template <> __device__ __forceinline__ uint32_t ld_data<uint32_t>(const uint32_t* p) {
+    return __ldcg(p);
+}
+template <> __device__ __forceinline__ int32_t ld_data<int32_t>(const int32_t* p) {
+    return __ldcg(p);
+}
+template <> __device__ __forceinline__ unsigned long long ld_data<unsigned long long>(
+    const unsigned long long* p) {
+    return __ldcg(p);
+}
+template <> __device__ __forceinline__ uint4 ld_data<uint4>(const uint4* p) { return __ldcg(p); }
+template <> __device__ __forceinline__ float ld_data<float>(const float* p) { return __ldcg(p); }
+template <> __device__ __forceinline__ double ld_data<double>(const double* p) {
+    return __ldcg(p);
+}
+
+__device__ __forceinline__ void set_err(const dev_cache* c, int code) {
+    atomicCAS(c->err, 0, code);
+}
+__device__ __forceinline__ dev_stats* my_stats(const dev_cache* c) {
+    return c->stats + (sm_id() % STAT_SHARDS);
+}
+__device__ __forceinline__ void stat_add(unsigned long long* ctr, unsigned long long v) {
+    if (v) atomicAdd(ctr, v);
+}
+
+/* k-th (0-based) set bit of m; m must have > k set bits. */
+__device__ __forceinline__ int nth_set(unsigned m, int k) {
+    for (int i = 0; i < k; ++i) m &= m - 1;
+    return __ffs(m) - 1;
+}
+
+/* -------------------------------------------------------------------------
+ * S10 unlink: lanes with `mine` drop their link to
+ * `page` of `r`.  Warp-aggregated: one release-add of -n per distinct page. */
+static __device__ AP_SLOW_ATTR void unlink_lanes(unsigned m, bool mine, const dev_region* r,
+                                          uint64_t page) {
+    unsigned long long key = mine ? (((unsigned long long)r->id << 48) | page) : ~0ull;
+    unsigned grp = __match_any_sync(m, key);
+    unsigned lane = lane_id();
+    if (mine && lane == (unsigned)(__ffs(grp) - 1)) {
+        unsigned n = __popc(grp);
+        red_add_release(r->pte + page, (uint64_t)0 - (uint64_t)n);
+        stat_add(&my_stats(r->cache)->unlinks, 1);
+    }
+}
+
+/* -------------------------------------------------------------------------
+ * S7 frame allocation, warp-cooperative.  Lanes with `want` need one frame
+ * each.  Free list first (pop-only array, R-A18), then victims: a warp-wide
+ * clock step examines 32 consecutive frames; a frame is a victim if its
+ * owner PTE is VALID, maps this frame and has reference count 0 (PAPER.md:
+ * 113, 145); the clock gives referenced pages a second chance (R-A11).  A
+ * victim is claimed by CAS of its PTE (VALID, rc=0) -> EMPTY, which a
+ * concurrent minor fault's CAS either precedes or loses to. */
+__device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, bool want,
+                                             uint32_t& frame) {
+    const unsigned lane = lane_id();
+    const int first = __ffs(m) - 1;
+    const unsigned wantm = __ballot_sync(m, want);
+    bool got = false;
+    {
+        const int k = __popc(wantm);
+        const int rank = __popc(wantm & lanemask_lt());
+        unsigned long long base = ~0ull;
+        if ((int)lane == first) {
+            if (*(volatile unsigned long long*)c->free_head < c->nfree)
+                base = atomicAdd(c->free_head, (unsigned long long)k);
+        }
+        base = __shfl_sync(m, base, first);
+        if (want && base != ~0ull && base + rank < c->nfree) {
+            frame = c->free_ids[base + rank];
+            got = true;
+        }
+    }
+    unsigned still = __ballot_sync(m, want && !got);
+    uint32_t steps = c->sweep_steps;
+    unsigned long long evicted = 0;
+    while (still && steps--) {
+        unsigned long long hb = 0;
+        if ((int)lane == first)
+            hb = atomicAdd(c->clock_hand, c->policy == POLICY_CLOCK ? 32ull : 1ull);
+        hb = __shfl_sync(m, hb, first);
+        uint64_t f;
+        if (c->policy == POLICY_CLOCK) f = (hb + lane) % c->frames;
+        else f = sm64(c->policy_seed ^ (hb << 5) ^ lane) % c->frames;
+        bool elig = false;
+        uint64_t e = 0;
+        uint64_t* q = nullptr;
+        const uint64_t own = ld_relaxed(c->owner + f);
+        if (own) {
+            const dev_region* vr = c->regions + ((own >> 48) - 1);
+            q = vr->pte + (own & PAGE_MASK48);
+            e = ld_relaxed(q);
+            if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f && (e & PTE_RC_MASK) == 0) {
+                if (c->policy == POLICY_CLOCK && (e & PTE_REF)) cas_acq_rel(q, e, e & ~PTE_REF);
+                else elig = true;
+            }
+        }
+        const unsigned cand = __ballot_sync(m, elig);
+        const int need_n = __popc(still);
+        bool won = false;
+        if (elig && __popc(cand & lanemask_lt()) < need_n) won = (cas_acq_rel(q, e, PTE_EMPTY) == e);
+        const unsigned wonm = __ballot_sync(m, won);
+        const int nwon = __popc(wonm);
+        evicted += nwon;
+        const bool mine_still = (still >> lane) & 1u;
+        const int srank = __popc(still & lanemask_lt());
+        const int src = (mine_still && srank < nwon) ? nth_set(wonm, srank) : (int)lane;
+        const uint32_t ff = __shfl_sync(m, (uint32_t)f, src);
+        if (mine_still && srank < nwon) {
+            frame = ff;
+            got = true;
+        }
+        still = __ballot_sync(m, want && !got);
+    }
+    if ((int)lane == first) {
+        stat_add(&my_stats(c)->evictions, evicted);
+        if (still) stat_add(&my_stats(c)->nofree, 1);
+    }
+    return got;
+}
+
+/* -------------------------------------------------------------------------
+ * S8 fill: the whole warp copies one page from pinned host memory (over the
+ * host link, zero-copy 16-B loads) into frame `f`; a ragged last page is
+ * zero-padded.  Host bytes are 16-B aligned (ap_mmap checks it). */
+__device__ __forceinline__ void fill_page(const dev_cache* c, const dev_region* r, uint64_t f,
+                                          uint64_t pg) {
+    const unsigned lane = lane_id();
+    const uint64_t P = 1ull << c->log2_page;
+    uint8_t* dst = c->pool + f * P;
+    const uint8_t* src = r->host + pg * P;
+    const uint64_t avail = r->bytes - pg * P;
+    const uint64_t len = avail < P ? avail : P;
+    const uint64_t nvec = len / 16;
+    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    uint4* d4 = reinterpret_cast<uint4*>(dst);
+    constexpr int U = 8;
+    uint64_t i = lane;
+    for (; i + 32 * (U - 1) < nvec; i += 32 * U) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = __ldcs(s4 + i + 32 * u);
+#pragma unroll
+        for (int u = 0; u < U; ++u) __stcg(d4 + i + 32 * u, v[u]);
+    }
+    for (; i < nvec; i += 32) __stcg(d4 + i, __ldcs(s4 + i));
+    if (len < P) {
+        /* ragged tail: bytes [nvec*16, len) from host, the rest zeros */
+        for (uint64_t b = nvec * 16 + lane; b < P; b += 32)
+            dst[b] = b < len ? src[b] : (uint8_t)0;
+    }
+}
+
+template <class T>
+struct slow_out {
+    uint64_t x;
+    uint64_t page;
+    T val;
+};
+
+/* -------------------------------------------------------------------------
+ * S5-S9: the fault handler (translation aggregation, Listing 1 / R-A9).
+ * Called by the converged lanes `m` when at least one of them is unlinked.
+ * Returns each lane's new translation and linked page; `val` receives the
+ * value at the lane's offset for lanes that were unlinked. */
+template <class T>
+__device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t page,
+                                               const dev_region* r, T val_in) {
+    T vv = val_in;
+    T* val = &vv;
+    const dev_cache* c = r->cache;
+    const unsigned lane = lane_id();
+    const uint32_t lg = c->log2_page;
+    const uint64_t P = 1ull << lg;
+    bool need = !(x >> 63);
+    if (need && (x + sizeof(T) > r->bytes || (x % sizeof(T)) != 0)) {
+        set_err(c, ERR_FAULT);
+        *val = T{};
+        need = false;
+    }
+    const uint64_t pg = need ? (x >> lg) : 0;
+    const unsigned long long mykey = ((unsigned long long)r->id << 48) | pg;
+    bool linked_here = false;
+    uint64_t t0 = 0;
+    uint32_t backoff = 64;
+    int idle_rounds = 0;
+    dev_stats* S = my_stats(c);
+
+    for (;;) {
+        const unsigned pend = __ballot_sync(m, need);
+        if (!pend) break;
+        const unsigned grp = __match_any_sync(m, need ? mykey : ~0ull);
+        const int leader = __ffs(grp) - 1;
+        const bool is_leader = need && (int)lane == leader;
+        const uint32_t n = __popc(grp);
+        uint64_t* pte = r->pte + pg;
+
+        /* Phase A (leaders, lane-parallel; R-A13): minor faults link at once;
+         * up to max_claims leaders (lane order) may claim an EMPTY entry. */
+        enum { ST_NONE = 0, ST_LINKED = 1, ST_CLAIMED = 2, ST_WAIT = 3, ST_SKIP = 4 };
+        int st = ST_NONE;
+        uint32_t frame = 0;
+        uint64_t old = is_leader ? ld_acquire(pte) : 0;
+        const unsigned empties = __ballot_sync(m, is_leader && (old >> 62) == 0);
+        const bool may_claim = !((empties >> lane) & 1u) ||
+                               (uint32_t)__popc(empties & lanemask_lt()) < c->max_claims;
+        if (is_leader) {
+            for (;;) {
+                const uint64_t s = old >> 62;
+                if (s == 2) {
+                    const uint64_t nw = (old + n) | PTE_REF;
+                    const uint64_t prev = cas_acq_rel(pte, old, nw);
+                    if (prev == old) {
+                        st = ST_LINKED;
+                        frame = (uint32_t)((old >> 32) & PTE_FRAME_MASK);
+                        break;
+                    }
+                    old = prev;
+                } else if (s == 0) {
+                    if (!may_claim) {
+                        st = ST_SKIP;
+                        break;
+                    }
+                    const uint64_t prev = cas_acq_rel(pte, old, PTE_LOADING);
+                    if (prev == old) {
+                        st = ST_CLAIMED;
+                        break;
+                    }
+                    old = prev;
+                } else {
+                    st = ST_WAIT;
+                    break;
+                }
+            }
+        }
+
+        /* Phase B: frames for the claimed pages (S7). */
+        const unsigned claimed = __ballot_sync(m, st == ST_CLAIMED);
+        if (claimed) {
+            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame);
+            if (st == ST_CLAIMED && !ok) {
+                st_release(pte, PTE_EMPTY); /* give the page back; retry later */
+                st = ST_WAIT;
+            }
+        }
+
+        /* Phase C: fills, one page at a time by the whole warp (S8), then the
+         * publish (S9): every lane fences its stores, the warp syncs, the
+         * leader release-stores VALID with the group's count. */
+        unsigned fill = __ballot_sync(m, st == ST_CLAIMED);
+        const int nfill = __popc(fill);
+        while (fill) {
+            const int L = __ffs(fill) - 1;
+            fill &= fill - 1;
+            const uint32_t f = __shfl_sync(m, frame, L);
+            const uint64_t fpg = __shfl_sync(m, pg, L);
+            const dev_region* fr =
+                reinterpret_cast<const dev_region*>(__shfl_sync(m, (unsigned long long)r, L));
+            if ((int)lane == L) st_relaxed(c->owner + f, ((uint64_t)(fr->id + 1) << 48) | fpg);
+            fill_page(c, fr, f, fpg);
+            fence_gpu();
+            __syncwarp(m);
+            if ((int)lane == L)
+                st_release(pte, PTE_VALID | PTE_REF | ((uint64_t)f << 32) | (uint64_t)n);
+        }
+        const unsigned nminor = __popc(__ballot_sync(m, st == ST_LINKED));
+
+        /* Phase D: link the group lanes and read their values (S9). */
+        const int lst = __shfl_sync(m, st, leader);
+        const uint32_t lf = __shfl_sync(m, frame, leader);
+        __syncwarp(m);
+        bool progressed = false;
+        if (need && (lst == ST_LINKED || lst == ST_CLAIMED)) {
+            x = XL_VALID | ((uint64_t)(c->pool + (uint64_t)lf * P) + (x & (P - 1)));
+            page = pg;
+            need = false;
+            linked_here = true;
+            *val = ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
+            progressed = true;
+        }
+        if ((int)lane == __ffs(m) - 1) {
+            stat_add(&S->major, nfill);
+            stat_add(&S->minor, nminor);
+        }
+        progressed = __any_sync(m, progressed);
+
+        /* Lanes still unserved: either skipped (another claim this round),
+         * waiting on a page another warp is loading, or out of frames. */
+        const unsigned waiting = __ballot_sync(m, need);
+        if (waiting) {
+            /* Under pressure (free list empty), stop pinning pages whose values
+             * are already in registers (PAPER.md:115 heuristic; R-A19). */
+            const bool pressure = *(volatile unsigned long long*)c->free_head >= c->nfree;
+            const bool waited = __any_sync(m, is_leader && st == ST_WAIT);
+            if (pressure || (waited && idle_rounds >= 2)) {
+                const bool dg = linked_here;
+                if (__any_sync(m, dg)) {
+                    unlink_lanes(m, dg, r, page);
+                    if (dg) {
+                        x = (page << lg) | (x & (P - 1));
+                        linked_here = false;
+                    }
+                    const unsigned ndg = __popc(__ballot_sync(m, dg));
+                    if ((int)lane == __ffs(m) - 1) stat_add(&S->downgrades, ndg);
+                }
+            }
+            if (!progressed) {
+                ++idle_rounds;
+                if ((int)lane == __ffs(m) - 1) stat_add(&S->waits, 1);
+                if (t0 == 0) t0 = now_ns();
+                else if (now_ns() - t0 > c->timeout_ns) {
+                    /* watchdog: give up on the remaining lanes (value 0). */
+                    if (need) {
+                        set_err(c, ERR_TIMEDOUT);
+                        *val = T{};
+                        need = false;
+                    }
+                    continue;
+                }
+                __nanosleep(backoff);
+                backoff = backoff < 4096 ? backoff * 2 : 4096;
+            } else {
+                idle_rounds = 0;
+                backoff = 64;
+                t0 = 0;
+            }
+        }
+    }
+    return slow_out<T>{x, page, vv};
+}
+
+}  // namespace detail
+
+/* ======================================================================
+ * ap::ptr<T> — the apointer (M1; Fig. 3).
+ * States: uninitialised (r == nullptr), unlinked (valid bit
+ * clear: x is the file offset), linked (valid bit set: x is the address of
+ * the datum in its frame, which is pinned by the page's reference count). */
+template <class T>
+struct ptr {
+    static_assert(sizeof(T) == 4 || sizeof(T) == 8 || sizeof(T) == 16, "T must be 4/8/16 B");
+    uint64_t x;
+    const dev_region* r;
+    uint64_t page;
+    uint32_t lg;
+
+    __device__ __forceinline__ ptr() : x(0), r(nullptr), page(0), lg(12) {}
+    __device__ __forceinline__ ptr(const dev_region* reg, uint32_t log2_page, uint64_t foff)
+        : x(foff), r(reg), page(0), lg(log2_page) {}
+    /* Copy: the copy starts unlinked (Fig. 4). */
+    __device__ __forceinline__ ptr(const ptr& o) : x(o.foff()), r(o.r), page(0), lg(o.lg) {}
+    __device__ __forceinline__ ptr& operator=(const ptr& o) {
+        const uint64_t nx = o.foff();
+        release();
+        x = nx;
+        r = o.r;
+        lg = o.lg;
+        return *this;
+    }
+    __device__ __forceinline__ ~ptr() { release(); }
+
+    __device__ __forceinline__ bool linked() const { return (x >> 63) != 0; }
+    /* File offset (xAddress) the pointer designates, linked or not. */
+    __device__ __forceinline__ uint64_t foff() const {
+        return linked() ? ((page << lg) | (x & ((1ull << lg) - 1))) : x;
+    }
+
+    /* S3: dereference (hit path inline, fault path out of line). */
+    __device__ __forceinline__ T operator*() {
+        const unsigned m = __activemask();
+        const bool v = linked();
+        const T* a = v ? reinterpret_cast<const T*>(x & XL_ADDR) : reinterpret_cast<const T*>(r);
+        T val = detail::ld_data<T>(a); /* speculative prefetch */
+        if (__all_sync(m, v)) return val;
+        const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r, val);
+        x = o.x;
+        page = o.page;
+        return o.val;
+    }
+
+    /* p[i] without moving p: a linked lane whose target stays in the page
+     * reads directly; otherwise a temporary pointer takes the fault. */
+    __device__ __forceinline__ T operator[](int64_t i) {
+        const unsigned m = __activemask();
+        const uint64_t nb = (uint64_t)(i * (int64_t)sizeof(T));
+        const uint64_t nx = x + nb;
+        const bool in = linked() && ((x ^ nx) >> lg) == 0;
+        const T* a = in ? reinterpret_cast<const T*>(nx & XL_ADDR) : reinterpret_cast<const T*>(r);
+        T val = detail::ld_data<T>(a);
+        if (__all_sync(m, in)) return val;
+        ptr q(*this);
+        q.x += nb;
+        return *q;
+    }
+
+    /* S4: arithmetic.  Staying inside the page keeps the link; leaving it
+     * unlinks with a warp-aggregated decrement (S10). */
+    __device__ __forceinline__ ptr& operator+=(int64_t d) {
+        const uint64_t nb = (uint64_t)(d * (int64_t)sizeof(T));
+        const uint64_t nx = x + nb;
+        const bool cross = linked() && ((x ^ nx) >> lg) != 0;
+        const unsigned m = __activemask();
+        if (__any_sync(m, cross)) {
+            detail::unlink_lanes(m, cross, r, page);
+            x = cross ? ((page << lg) | (x & ((1ull << lg) - 1))) + nb : nx;
+        } else {
+            x = nx;
+        }
+        return *this;
+    }
+    __device__ __forceinline__ ptr& operator-=(int64_t d) { return *this += -d; }
+    __device__ __forceinline__ ptr& operator++() { return *this += 1; }
+    __device__ __forceinline__ ptr& operator--() { return *this += -1; }
+    /* p + d is a new, unlinked pointer. */
+    __device__ __forceinline__ ptr operator+(int64_t d) const {
+        ptr q(*this);
+        q.x += (uint64_t)(d * (int64_t)sizeof(T));
+        return q;
+    }
+
+    /* Unlink now (also done by the destructor and by assignment). */
+    __device__ __forceinline__ void release() {
+        const unsigned m = __activemask();
+        const bool l = linked();
+        if (__any_sync(m, l)) {
+            detail::unlink_lanes(m, l, r, page);
+            if (l) x = (page << lg) | (x & ((1ull << lg) - 1));
+        }
+    }
+};
+
+/* gvmmap (M17): an unlinked apointer to byte offset
+ * `foff` of region `region` of the cache.  Read-only mappings only. */
+template <class T>
+__device__ __forceinline__ ptr<T> gvmmap(const dev_cache* c, uint32_t region, uint64_t foff) {
+    return ptr<T>(c->regions + region, c->log2_page, foff);
+}
+
+}  // namespace ap
+
+#endif /* AP_APOINTER_CUH_ */

@@ -1,0 +1,182 @@
+"""ActivePointers on B200 -- Python binding of libapointer.so (include/ap.h).
+
+Same names as the C ABI; arguments are marshalled, nothing is computed here.
+Device buffers are torch CUDA tensors (PyTorch provides memory and streams
+only); host buffers are numpy arrays or torch CPU tensors.
+"""
+import ctypes
+
+import numpy as np
+
+from . import _lib
+from ._lib import (AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK,  # noqa: F401
+                   AP_POLICY_RANDOM, AP_SEQ, AP_UNIFORM, APError, ap_bench_cfg, ap_collage_in,
+                   ap_stats_t)
+
+_frames = {}
+
+
+def _ptr(buf):
+    """Address of a numpy array / torch tensor / raw int."""
+    if buf is None:
+        return None
+    if isinstance(buf, int):
+        return buf
+    if isinstance(buf, np.ndarray):
+        return buf.ctypes.data
+    if hasattr(buf, "data_ptr"):
+        return buf.data_ptr()
+    raise TypeError(f"cannot take the address of {type(buf)}")
+
+
+def _nbytes(buf):
+    if isinstance(buf, np.ndarray):
+        return buf.nbytes
+    if hasattr(buf, "element_size"):
+        return buf.numel() * buf.element_size()
+    raise TypeError(type(buf))
+
+
+def _stream(stream):
+    if stream is None:
+        try:
+            import torch
+            if torch.cuda.is_available():
+                return torch.cuda.current_stream().cuda_stream
+        except Exception:
+            pass
+        return None
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def ap_version():
+    return _lib.lib().ap_version().decode()
+
+
+def ap_strerror(code):
+    return _lib.lib().ap_strerror(code).decode()
+
+
+def ap_cache_create(frames, page_size, device=0):
+    h = ctypes.c_void_p()
+    _lib.check("ap_cache_create", _lib.lib().ap_cache_create(frames, page_size, device,
+                                                             ctypes.byref(h)))
+    _frames[h.value] = frames
+    return h.value
+
+
+def ap_cache_destroy(cache):
+    _lib.check("ap_cache_destroy", _lib.lib().ap_cache_destroy(cache))
+    _frames.pop(cache, None)
+
+
+def ap_mmap(cache, host_buf, nbytes=None):
+    r = ctypes.c_uint32()
+    nbytes = _nbytes(host_buf) if nbytes is None else nbytes
+    _lib.check("ap_mmap", _lib.lib().ap_mmap(cache, _ptr(host_buf), nbytes, ctypes.byref(r)))
+    return r.value
+
+
+def ap_munmap(cache, region):
+    _lib.check("ap_munmap", _lib.lib().ap_munmap(cache, region))
+
+
+def ap_region_devptr(cache, region):
+    p = ctypes.c_void_p()
+    _lib.check("ap_region_devptr", _lib.lib().ap_region_devptr(cache, region, ctypes.byref(p)))
+    return p.value
+
+
+def ap_region_npages(cache, region):
+    n = ctypes.c_uint64()
+    _lib.check("ap_region_npages", _lib.lib().ap_region_npages(cache, region, ctypes.byref(n)))
+    return n.value
+
+
+def ap_cache_stats(cache):
+    s = ap_stats_t()
+    _lib.check("ap_cache_stats", _lib.lib().ap_cache_stats(cache, ctypes.byref(s)))
+    return s.as_dict()
+
+
+def ap_cache_reset(cache):
+    _lib.check("ap_cache_reset", _lib.lib().ap_cache_reset(cache))
+
+
+def ap_cache_set_policy(cache, policy, seed=0):
+    _lib.check("ap_cache_set_policy", _lib.lib().ap_cache_set_policy(cache, policy, seed))
+
+
+def ap_cache_set_tuning(cache, max_claims=1, sweep_steps=64, timeout_ms=0):
+    _lib.check("ap_cache_set_tuning",
+               _lib.lib().ap_cache_set_tuning(cache, max_claims, sweep_steps, timeout_ms))
+
+
+def ap_last_device_error(cache):
+    return _lib.lib().ap_last_device_error(cache)
+
+
+def ap_cache_dump(cache):
+    frames = _frames[cache]
+    owner = np.empty(frames, dtype=np.uint64)
+    left = ctypes.c_uint64()
+    _lib.check("ap_cache_dump", _lib.lib().ap_cache_dump(cache, owner.ctypes.data,
+                                                         ctypes.byref(left)))
+    return owner, left.value
+
+
+def ap_region_dump_pte(cache, region):
+    pte = np.empty(ap_region_npages(cache, region), dtype=np.uint64)
+    _lib.check("ap_region_dump_pte", _lib.lib().ap_region_dump_pte(cache, region,
+                                                                   pte.ctypes.data))
+    return pte
+
+
+def ap_prefill(cache, region, first_page, npages, stream=None):
+    _lib.check("ap_prefill", _lib.lib().ap_prefill(cache, region, first_page, npages,
+                                                   _stream(stream)))
+
+
+def bench_cfg(pattern, elem_bytes, grid, block, reads_per_thread=0, passes=1, unit_bytes=0,
+              page_bytes=0, span_bytes=0, seed=0, mode=AP_MODE_APOINTER, out_copy=False,
+              raw_base=None):
+    return ap_bench_cfg(pattern, elem_bytes, grid, block, reads_per_thread, passes, unit_bytes,
+                        page_bytes, span_bytes, seed, mode, int(out_copy), raw_base)
+
+
+def ap_bench_read(cache, region, cfg, out_dev, stream=None):
+    _lib.check("ap_bench_read", _lib.lib().ap_bench_read(cache, region, ctypes.byref(cfg),
+                                                         _ptr(out_dev), _stream(stream)))
+
+
+def ap_bench_read_host(cache, region, cfg, out_host):
+    sec = ctypes.c_double()
+    _lib.check("ap_bench_read_host", _lib.lib().ap_bench_read_host(
+        cache, region, ctypes.byref(cfg), _ptr(out_host), ctypes.byref(sec)))
+    return sec.value
+
+
+def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev, ids_dev, N,
+               rec_stride=4096, group=1, block_begin=0, block_count=None,
+               mode=AP_MODE_APOINTER, raw_base=None, L=None, K=None):
+    L = proj_dev.shape[0] if L is None else L
+    K = proj_dev.shape[1] if K is None else K
+    nb = (W // 32) * (H // 32)
+    block_count = nb - block_begin if block_count is None else block_count
+    return ap_collage_in(_ptr(target_dev), W, H, L, K, bucket_bits, w, _ptr(proj_dev),
+                         _ptr(bias_dev), _ptr(offsets_dev), _ptr(ids_dev), N, rec_stride, group,
+                         block_begin, block_count, mode, _ptr(raw_base))
+
+
+def ap_collage_run(cache, region, inp, winners_dev, stream=None):
+    _lib.check("ap_collage_run", _lib.lib().ap_collage_run(cache, region, ctypes.byref(inp),
+                                                           _ptr(winners_dev), _stream(stream)))
+
+
+def ap_lsh_build_index(cache, region, N, rec_stride, L, K, bucket_bits, w, proj_dev, bias_dev,
+                       offsets_dev, ids_dev, stream=None):
+    _lib.check("ap_lsh_build_index", _lib.lib().ap_lsh_build_index(
+        cache, region, N, rec_stride, L, K, bucket_bits, w, _ptr(proj_dev), _ptr(bias_dev),
+        _ptr(offsets_dev), _ptr(ids_dev), _stream(stream)))

@@ -1,0 +1,104 @@
+"""ctypes binding of libapointer.so (include/ap.h). Argument marshalling only:
+every step of the path runs in the library's CUDA kernels.
+
+Fails loudly when the library is missing -- there is no CPU fallback.
+"""
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libapointer.so")
+
+AP_OK = 0
+AP_EINVAL, AP_ENOMEM, AP_ECUDA, AP_EBUSY, AP_ERANGE = -1, -2, -3, -4, -5
+AP_EFAULT, AP_ENOFRAME, AP_ETIMEDOUT = -6, -7, -8
+AP_POLICY_CLOCK, AP_POLICY_RANDOM = 0, 1
+AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
+AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
+
+u64, u32, i32, vp, ci = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int
+
+
+class ap_stats_t(ctypes.Structure):
+    _fields_ = [(n, u64) for n in ("major", "minor", "fill_bytes", "evictions", "waits",
+                                   "downgrades", "nofree", "unlinks")]
+
+    def as_dict(self):
+        return {n: int(getattr(self, n)) for n, _ in self._fields_}
+
+
+class ap_bench_cfg(ctypes.Structure):
+    _fields_ = [("pattern", i32), ("elem_bytes", u32), ("grid", u32), ("block", u32),
+                ("reads_per_thread", u32), ("passes", u32), ("unit_bytes", u32),
+                ("page_bytes", u32), ("span_bytes", u64), ("seed", u64), ("mode", i32),
+                ("out_copy", i32), ("raw_base", vp)]
+
+
+class ap_collage_in(ctypes.Structure):
+    _fields_ = [("target_dev", vp), ("W", u32), ("H", u32), ("L", u32), ("K", u32),
+                ("bucket_bits", u32), ("w", i32), ("proj_dev", vp), ("bias_dev", vp),
+                ("offsets_dev", vp), ("ids_dev", vp), ("N", u64), ("rec_stride", u32),
+                ("group", u32), ("block_begin", u64), ("block_count", u64), ("mode", i32),
+                ("raw_base", vp)]
+
+
+class APError(RuntimeError):
+    def __init__(self, fn, code, msg):
+        super().__init__(f"{fn} failed: {code} ({msg})")
+        self.code = code
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(
+                f"{LIB_PATH} is missing: the CUDA extension must be built (`make` or "
+                f"__graft_entry__.build()); there is no fallback path")
+        L = ctypes.CDLL(LIB_PATH)
+        sig = {
+            "ap_strerror": (ctypes.c_char_p, [ci]),
+            "ap_version": (ctypes.c_char_p, []),
+            "ap_cache_create": (ci, [u64, u32, ci, ctypes.POINTER(vp)]),
+            "ap_cache_destroy": (ci, [vp]),
+            "ap_mmap": (ci, [vp, vp, u64, ctypes.POINTER(u32)]),
+            "ap_munmap": (ci, [vp, u32]),
+            "ap_region_devptr": (ci, [vp, u32, ctypes.POINTER(vp)]),
+            "ap_region_npages": (ci, [vp, u32, ctypes.POINTER(u64)]),
+            "ap_cache_stats": (ci, [vp, ctypes.POINTER(ap_stats_t)]),
+            "ap_cache_reset": (ci, [vp]),
+            "ap_cache_set_policy": (ci, [vp, ci, u64]),
+            "ap_cache_set_tuning": (ci, [vp, u32, u32, u32]),
+            "ap_last_device_error": (ci, [vp]),
+            "ap_cache_dump": (ci, [vp, vp, ctypes.POINTER(u64)]),
+            "ap_region_dump_pte": (ci, [vp, u32, vp]),
+            "ap_prefill": (ci, [vp, u32, u64, u64, vp]),
+            "ap_bench_read": (ci, [vp, u32, ctypes.POINTER(ap_bench_cfg), vp, vp]),
+            "ap_bench_read_host": (ci, [vp, u32, ctypes.POINTER(ap_bench_cfg), vp,
+                                        ctypes.POINTER(ctypes.c_double)]),
+            "ap_collage_run": (ci, [vp, u32, ctypes.POINTER(ap_collage_in), vp, vp]),
+            "ap_lsh_build_index": (ci, [vp, u32, u64, u32, u32, u32, u32, i32, vp, vp, vp, vp,
+                                        vp]),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", "ap_mmap",
+            "ap_munmap", "ap_region_devptr", "ap_region_npages", "ap_cache_stats",
+            "ap_cache_reset", "ap_cache_set_policy", "ap_cache_set_tuning",
+            "ap_last_device_error", "ap_cache_dump", "ap_region_dump_pte", "ap_prefill",
+            "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index"]
+
+
+def check(fn, rc):
+    if rc != AP_OK:
+        raise APError(fn, rc, lib().ap_strerror(rc).decode())
+    return rc

@@ -1,0 +1,286 @@
+/*
+ * ap_bench.cu — the apointer microbenchmarks (§VI-A/C) on
+ * B200, each in two versions that differ only in the pointer type
+ * ("We develop two versions of every benchmark"):
+ *
+ *   SEQ        warp w sweeps units w, w+W, ... of the file; lanes read
+ *              consecutive elements (coalesced), `q += 32` between reads
+ *              (the copy/throughput kernel, and the page
+ *              walk of PAPER.md:367 "each warp accesses ... different pages in
+ *              a loop, with all threads in a warp accessing the same page").
+ *   UNIFORM    uniform-random element offsets, reached by pointer arithmetic
+ *              from the previous offset (C2).
+ *   DIVERGENT  the 32 lanes of a warp on 32 distinct pages (C3).
+ *
+ * Output: per-thread FNV-1a-64 over the values read (or the bytes themselves
+ * for SEQ out_copy).  Workload definitions: DESIGN.md "Workloads".
+ */
+#include <cuda_runtime.h>
+
+#include "ap_internal.cuh"
+
+/* The apointer kernels need ~120 registers once the fault path is linked
+ * in; 512 threads x 128 registers = one CTA of 16 warps per SM. */
+#ifndef AP_BENCH_THREADS
+#define AP_BENCH_THREADS 512
+#endif
+#ifndef AP_BENCH_MINB
+#define AP_BENCH_MINB 1
+#endif
+
+namespace {
+
+constexpr uint64_t FNV_BASIS = 0xcbf29ce484222325ull;
+constexpr uint64_t FNV_PRIME = 0x100000001b3ull;
+
+__device__ __forceinline__ uint64_t fnv(uint64_t h, uint32_t v) {
+    return (h ^ (uint64_t)v) * FNV_PRIME;
+}
+__device__ __forceinline__ uint64_t fnv(uint64_t h, unsigned long long v) {
+    return (h ^ (uint64_t)v) * FNV_PRIME;
+}
+__device__ __forceinline__ uint64_t fnv(uint64_t h, uint4 v) {
+    h = (h ^ (((uint64_t)v.y << 32) | v.x)) * FNV_PRIME;
+    return (h ^ (((uint64_t)v.w << 32) | v.z)) * FNV_PRIME;
+}
+
+struct BenchArgs {
+    uint64_t bytes;     /* region bytes                                 */
+    uint64_t span;      /* SEQ sweep bytes                              */
+    uint32_t unit;      /* SEQ unit bytes                               */
+    uint32_t passes;    /* SEQ                                          */
+    uint32_t reads;     /* UNIFORM / DIVERGENT                          */
+    uint32_t page;      /* DIVERGENT pattern page size                  */
+    uint64_t seed;
+    const uint8_t* raw; /* RAW twin base                                */
+    uint8_t* out_copy;  /* SEQ copy output or nullptr                   */
+    uint64_t* ck;       /* per-thread checksums                         */
+};
+
+__device__ __forceinline__ uint64_t uniform_off(const BenchArgs& a, uint32_t E, uint64_t t,
+                                                uint64_t i) {
+    return (ap::detail::sm64(a.seed ^ (t << 24) ^ i) % (a.bytes / E)) * E;
+}
+
+__device__ __forceinline__ uint64_t divergent_off(const BenchArgs& a, uint32_t E, uint64_t t,
+                                                  uint64_t i) {
+    const uint64_t npg = a.bytes / a.page;
+    const uint64_t w = t >> 5, lane = t & 31;
+    const uint64_t pg = (ap::detail::sm64(a.seed ^ (w << 24) ^ i) + lane * (npg / 32)) % npg;
+    const uint64_t el =
+        ap::detail::sm64(a.seed ^ (t << 24) ^ i ^ 0xD1B54A32D192ED03ull) % (a.page / E);
+    return pg * a.page + el * E;
+}
+
+/* ------------------------------------------------------------ SEQ */
+/* Loads are tiled TILE deep ("memory tiling ... interleaves
+ * memory copy operations"): TILE dereferences are issued before the values
+ * are consumed, so each warp keeps TILE requests in flight. */
+constexpr int TILE = 8;
+
+template <class T>
+__device__ __forceinline__ void consume(const BenchArgs& a, uint64_t off, const T& v,
+                                        uint64_t& h) {
+    if (a.out_copy) *reinterpret_cast<T*>(a.out_copy + off) = v;
+    else h = fnv(h, v);
+}
+
+template <class T, bool APTR>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
+    k_seq(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t w = t >> 5, lane = t & 31;
+    const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
+    const uint32_t per_unit = a.unit / (32 * E);
+    uint64_t h = FNV_BASIS;
+    for (uint32_t pass = 0; pass < a.passes; ++pass) {
+        for (uint64_t u = w; u < nunits; u += W) {
+            const uint64_t e0 = u * (a.unit / E) + lane;
+            /* whole unit inside the span: tiled fast loop; else per element */
+            const bool whole = (u + 1) * a.unit <= a.span;
+            if constexpr (APTR) {
+                ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
+                uint32_t j = 0;
+                if (whole) {
+                    for (; j + TILE <= per_unit; j += TILE) {
+                        T v[TILE];
+#pragma unroll
+                        for (int k = 0; k < TILE; ++k) {
+                            v[k] = *q;
+                            q += 32;
+                        }
+#pragma unroll
+                        for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
+                    }
+                }
+                for (; j < per_unit; ++j) {
+                    const uint64_t off = (e0 + 32ull * j) * E;
+                    if (off + E <= a.span) consume(a, off, (T)*q, h);
+                    q += 32;
+                }
+            } else {
+                const T* q = reinterpret_cast<const T*>(a.raw) + e0;
+                uint32_t j = 0;
+                if (whole) {
+                    for (; j + TILE <= per_unit; j += TILE) {
+                        T v[TILE];
+#pragma unroll
+                        for (int k = 0; k < TILE; ++k) {
+                            v[k] = ap::detail::ld_data<T>(q);
+                            q += 32;
+                        }
+#pragma unroll
+                        for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
+                    }
+                }
+                for (; j < per_unit; ++j) {
+                    const uint64_t off = (e0 + 32ull * j) * E;
+                    if (off + E <= a.span) consume(a, off, ap::detail::ld_data<T>(q), h);
+                    q += 32;
+                }
+            }
+        }
+    }
+    if (!a.out_copy) a.ck[t] = h;
+}
+
+/* ------------------------------------------------------------ UNIFORM / DIVERGENT */
+template <class T, int PAT, bool APTR>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
+    k_random(const ap::dev_cache* __restrict__ c,
+                                                  uint32_t region, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint64_t h = FNV_BASIS;
+    if constexpr (APTR) {
+        ap::ptr<T> p = ap::gvmmap<T>(c, region, 0);
+        uint64_t cur = 0;
+        for (uint32_t i = 0; i < a.reads; ++i) {
+            const uint64_t off = PAT == AP_UNIFORM ? uniform_off(a, E, t, i)
+                                                   : divergent_off(a, E, t, i);
+            p += ((int64_t)off - (int64_t)cur) / (int64_t)E; /* pointer arithmetic (S4) */
+            cur = off;
+            h = fnv(h, *p);
+        }
+    } else {
+        const T* base = reinterpret_cast<const T*>(a.raw);
+        for (uint32_t i = 0; i < a.reads; ++i) {
+            const uint64_t off = PAT == AP_UNIFORM ? uniform_off(a, E, t, i)
+                                                   : divergent_off(a, E, t, i);
+            h = fnv(h, ap::detail::ld_data<T>(base + off / E));
+        }
+    }
+    a.ck[t] = h;
+}
+
+template <class T, bool APTR>
+cudaError_t launch_t(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg,
+                     const BenchArgs& a, cudaStream_t s) {
+    switch (cfg->pattern) {
+        case AP_SEQ: k_seq<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a); break;
+        case AP_UNIFORM:
+            k_random<T, AP_UNIFORM, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            break;
+        default:
+            k_random<T, AP_DIVERGENT, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region,
+                                                                              a);
+    }
+    return cudaGetLastError();
+}
+
+template <bool APTR>
+cudaError_t launch_m(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg,
+                     const BenchArgs& a, cudaStream_t s) {
+    switch (cfg->elem_bytes) {
+        case 4: return launch_t<uint32_t, APTR>(c, region, cfg, a, s);
+        case 8: return launch_t<unsigned long long, APTR>(c, region, cfg, a, s);
+        default: return launch_t<uint4, APTR>(c, region, cfg, a, s);
+    }
+}
+
+int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, void* out,
+              BenchArgs* a) {
+    if (!ap_region_ok(c, region) || !cfg || !out) return AP_EINVAL;
+    const uint32_t E = cfg->elem_bytes;
+    if (E != 4 && E != 8 && E != 16) return AP_EINVAL;
+    if (cfg->grid == 0 || cfg->block == 0 || cfg->block > AP_BENCH_THREADS || cfg->block % 32)
+        return AP_EINVAL;
+    if (cfg->mode != AP_MODE_APOINTER && cfg->mode != AP_MODE_RAW) return AP_EINVAL;
+    if (cfg->mode == AP_MODE_RAW && !cfg->raw_base) return AP_EINVAL;
+    const ap_region_host& rg = c->reg[region];
+    *a = BenchArgs{};
+    a->bytes = rg.bytes;
+    a->seed = cfg->seed;
+    a->raw = (const uint8_t*)cfg->raw_base;
+    a->reads = cfg->reads_per_thread;
+    a->passes = cfg->passes;
+    a->unit = cfg->unit_bytes;
+    a->page = cfg->page_bytes;
+    a->span = cfg->span_bytes ? cfg->span_bytes : rg.bytes;
+    switch (cfg->pattern) {
+        case AP_SEQ:
+            if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;
+            if (cfg->mode == AP_MODE_APOINTER && (c->page % a->unit)) return AP_EINVAL;
+            if (cfg->out_copy) a->out_copy = (uint8_t*)out;
+            else a->ck = (uint64_t*)out;
+            break;
+        case AP_UNIFORM:
+            if (rg.bytes < E) return AP_EINVAL;
+            a->ck = (uint64_t*)out;
+            break;
+        case AP_DIVERGENT:
+            if (a->page == 0 || (a->page & (a->page - 1)) || a->page < E ||
+                rg.bytes / a->page < 32)
+                return AP_EINVAL;
+            a->ck = (uint64_t*)out;
+            break;
+        default: return AP_EINVAL;
+    }
+    return AP_OK;
+}
+
+}  // namespace
+
+extern "C" int ap_bench_read(ap_cache_t c, ap_region_t region, const ap_bench_cfg* cfg,
+                             void* out_dev, void* stream) {
+    BenchArgs a;
+    int rc = make_args(c, region, cfg, out_dev, &a);
+    if (rc) return rc;
+    ap_device_guard g(c->device);
+    cudaError_t e = cfg->mode == AP_MODE_APOINTER
+                        ? launch_m<true>(c, region, cfg, a, (cudaStream_t)stream)
+                        : launch_m<false>(c, region, cfg, a, (cudaStream_t)stream);
+    AP_CUDA_TRY(e);
+    return AP_OK;
+}
+
+extern "C" int ap_bench_read_host(ap_cache_t c, ap_region_t region, const ap_bench_cfg* cfg,
+                                  void* out_host, double* seconds) {
+    if (!c || !cfg || !out_host) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    const uint64_t nthreads = (uint64_t)cfg->grid * cfg->block;
+    uint64_t out_bytes = nthreads * 8;
+    if (cfg->pattern == AP_SEQ && cfg->out_copy)
+        out_bytes = cfg->span_bytes ? cfg->span_bytes : c->reg[region].bytes;
+    void* d = nullptr;
+    AP_CUDA_TRY(cudaMalloc(&d, out_bytes));
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    cudaEventRecord(e0, 0);
+    int rc = ap_bench_read(c, region, cfg, d, nullptr);
+    if (rc == AP_OK) {
+        cudaMemcpyAsync(out_host, d, out_bytes, cudaMemcpyDeviceToHost, 0);
+        cudaEventRecord(e1, 0);
+        if (cudaEventSynchronize(e1) != cudaSuccess) rc = AP_ECUDA;
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (seconds) *seconds = ms * 1e-3;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(d);
+    return rc;
+}

@@ -1,0 +1,71 @@
+/* ap_internal.cuh — host-side state of a cache, shared by the library's
+ * translation units (runtime, benchmarks, collage).  Not installed. */
+#ifndef AP_INTERNAL_CUH_
+#define AP_INTERNAL_CUH_
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <vector>
+
+#include "ap.h"
+#include "ap/apointer.cuh"
+
+constexpr uint32_t AP_MAX_REGIONS = 65535;
+
+struct ap_region_host {
+    const void* host_buf = nullptr; /* caller's pointer                      */
+    const uint8_t* dev_alias = nullptr;
+    uint64_t bytes = 0;
+    uint64_t npages = 0;
+    uint64_t* pte = nullptr; /* device                                     */
+    bool registered = false; /* we called cudaHostRegister                 */
+    bool live = false;
+};
+
+struct ap_cache_s {
+    int device = 0;
+    uint64_t frames = 0;
+    uint32_t page = 0, log2_page = 0;
+    void* pool_raw = nullptr;
+    uint8_t* pool = nullptr;
+    uint64_t* owner = nullptr;
+    uint32_t* free_ids = nullptr;
+    unsigned long long* free_head = nullptr;
+    unsigned long long* clock_hand = nullptr;
+    ap::dev_region* regions = nullptr;
+    ap::dev_stats* stats = nullptr;
+    int* err = nullptr;
+    ap::dev_cache* d_cache = nullptr; /* device copy of `h` */
+    ap::dev_cache h{};                /* host mirror         */
+    std::vector<ap_region_host> reg;
+    int num_sms = 148;
+};
+
+/* Switch to the cache's device for the lifetime of the guard. */
+struct ap_device_guard {
+    int prev = -1;
+    explicit ap_device_guard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~ap_device_guard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+#define AP_CUDA_TRY(expr)                                  \
+    do {                                                   \
+        cudaError_t e__ = (expr);                          \
+        if (e__ != cudaSuccess) {                          \
+            ap_note_cuda_error(e__, #expr, __FILE__, __LINE__); \
+            return AP_ECUDA;                               \
+        }                                                  \
+    } while (0)
+
+void ap_note_cuda_error(cudaError_t e, const char* what, const char* file, int line);
+bool ap_region_ok(const ap_cache_s* c, ap_region_t r);
+
+#endif

@@ -1,0 +1,408 @@
+/*
+ * ap_runtime.cu — host runtime of the apointer library: the page cache
+ * (§V), file mapping (gvmmap, PAPER.md:125/131/367),
+ * statistics, reset, dumps, prefill.  C ABI in include/ap.h.
+ */
+#include <cuda_runtime.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "ap_internal.cuh"
+
+void ap_note_cuda_error(cudaError_t e, const char* what, const char* file, int line) {
+    if (getenv("AP_VERBOSE"))
+        fprintf(stderr, "[ap] %s:%d: %s -> %s\n", file, line, what, cudaGetErrorString(e));
+}
+
+extern "C" const char* ap_strerror(int code) {
+    switch (code) {
+        case AP_OK: return "ok";
+        case AP_EINVAL: return "invalid argument";
+        case AP_ENOMEM: return "out of memory";
+        case AP_ECUDA: return "CUDA runtime error";
+        case AP_EBUSY: return "busy: live references or mapped regions";
+        case AP_ERANGE: return "out of range";
+        case AP_EFAULT: return "device: dereference outside the mapped region or misaligned";
+        case AP_ENOFRAME: return "device: no evictable frame";
+        case AP_ETIMEDOUT: return "device: fault-path watchdog expired";
+        default: return "unknown error";
+    }
+}
+
+extern "C" const char* ap_version(void) {
+    return "apointer-b200 0.1 (sm_100a; long apointer, no TLB, clock eviction)";
+}
+
+bool ap_region_ok(const ap_cache_s* c, ap_region_t r) {
+    return c && r < c->reg.size() && c->reg[r].live;
+}
+
+static int push_descriptor(ap_cache_s* c) {
+    AP_CUDA_TRY(cudaMemcpy(c->d_cache, &c->h, sizeof(ap::dev_cache), cudaMemcpyHostToDevice));
+    return AP_OK;
+}
+
+/* ------------------------------------------------------------ kernels */
+__global__ void k_iota(uint32_t* a, uint64_t n) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        a[i] = (uint32_t)i;
+}
+
+/* flag bit0: a positive reference count; bit1: an entry left LOADING. */
+__global__ void k_scan_pte(const uint64_t* pte, uint64_t n, int* flag) {
+    int f = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t e = pte[i];
+        if (e & ap::PTE_RC_MASK) f |= 1;
+        if ((e >> 62) == 1) f |= 2;
+    }
+    if (f) atomicOr(flag, f);
+}
+
+__global__ void k_drop_owner(uint64_t* owner, uint64_t frames, uint64_t tag) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < frames;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        if ((owner[i] >> 48) == tag) owner[i] = 0;
+}
+
+/* One warp per page: an apointer dereference faults it in; the pointer is
+ * destroyed at scope exit, leaving the page resident with count 0. */
+__global__ void k_prefill(const ap::dev_cache* __restrict__ c, uint32_t region, uint64_t first,
+                          uint64_t npages) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) / 32;
+    const uint64_t nwarps = (uint64_t)gridDim.x * blockDim.x / 32;
+    const uint32_t lg = c->log2_page;
+    for (uint64_t p = first + warp; p < first + npages; p += nwarps) {
+        ap::ptr<uint32_t> q = ap::gvmmap<uint32_t>(c, region, p << lg);
+        volatile uint32_t v = *q;
+        (void)v;
+    }
+}
+
+static int scan_refs(ap_cache_s* c, const ap_region_host& rg, int* result) {
+    int* d_flag = nullptr;
+    AP_CUDA_TRY(cudaMalloc(&d_flag, sizeof(int)));
+    AP_CUDA_TRY(cudaMemset(d_flag, 0, sizeof(int)));
+    k_scan_pte<<<c->num_sms * 4, 256>>>(rg.pte, rg.npages, d_flag);
+    int h = 0;
+    cudaError_t e = cudaMemcpy(&h, d_flag, sizeof(int), cudaMemcpyDeviceToHost);
+    cudaFree(d_flag);
+    AP_CUDA_TRY(e);
+    *result = h;
+    return AP_OK;
+}
+
+/* Free list = every frame without an owner, ascending (R-A18). */
+static int rebuild_free_list(ap_cache_s* c) {
+    std::vector<uint64_t> owner(c->frames);
+    AP_CUDA_TRY(cudaMemcpy(owner.data(), c->owner, c->frames * 8, cudaMemcpyDeviceToHost));
+    std::vector<uint32_t> ids;
+    ids.reserve(c->frames);
+    for (uint64_t f = 0; f < c->frames; ++f)
+        if (owner[f] == 0) ids.push_back((uint32_t)f);
+    if (!ids.empty())
+        AP_CUDA_TRY(cudaMemcpy(c->free_ids, ids.data(), ids.size() * 4, cudaMemcpyHostToDevice));
+    AP_CUDA_TRY(cudaMemset(c->free_head, 0, sizeof(unsigned long long)));
+    c->h.nfree = ids.size();
+    return push_descriptor(c);
+}
+
+/* ------------------------------------------------------------ the cache */
+extern "C" int ap_cache_create(uint64_t frames, uint32_t page_size, int device, ap_cache_t* out) {
+    if (!out || frames == 0 || frames > ap::PTE_FRAME_MASK) return AP_EINVAL;
+    if (page_size < 4096 || page_size > (2u << 20) || (page_size & (page_size - 1))) return AP_EINVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return AP_EINVAL;
+    ap_device_guard g(device);
+    ap_cache_s* c = new ap_cache_s();
+    c->device = device;
+    c->frames = frames;
+    c->page = page_size;
+    c->log2_page = 0;
+    while ((1u << c->log2_page) < page_size) ++c->log2_page;
+    cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
+    auto fail = [&](int code) {
+        cudaFree(c->pool_raw);
+        cudaFree(c->owner);
+        cudaFree(c->free_ids);
+        cudaFree(c->free_head);
+        cudaFree(c->regions);
+        cudaFree(c->stats);
+        cudaFree(c->d_cache);
+        delete c;
+        cudaGetLastError();
+        return code;
+    };
+    const uint64_t pool_bytes = frames * (uint64_t)page_size + page_size;
+    if (cudaMalloc(&c->pool_raw, pool_bytes) != cudaSuccess) return fail(AP_ENOMEM);
+    c->pool = (uint8_t*)(((uintptr_t)c->pool_raw + page_size - 1) & ~(uintptr_t)(page_size - 1));
+    if (cudaMalloc(&c->owner, frames * 8) != cudaSuccess) return fail(AP_ENOMEM);
+    if (cudaMalloc(&c->free_ids, frames * 4) != cudaSuccess) return fail(AP_ENOMEM);
+    /* free_head, clock_hand and err share one small allocation */
+    if (cudaMalloc(&c->free_head, 256) != cudaSuccess) return fail(AP_ENOMEM);
+    c->clock_hand = c->free_head + 8;
+    c->err = (int*)(c->free_head + 16);
+    if (cudaMalloc(&c->regions, sizeof(ap::dev_region) * AP_MAX_REGIONS) != cudaSuccess)
+        return fail(AP_ENOMEM);
+    if (cudaMalloc(&c->stats, sizeof(ap::dev_stats) * ap::STAT_SHARDS) != cudaSuccess)
+        return fail(AP_ENOMEM);
+    if (cudaMalloc(&c->d_cache, sizeof(ap::dev_cache)) != cudaSuccess) return fail(AP_ENOMEM);
+    if (cudaMemset(c->owner, 0, frames * 8) != cudaSuccess ||
+        cudaMemset(c->free_head, 0, 256) != cudaSuccess ||
+        cudaMemset(c->regions, 0, sizeof(ap::dev_region) * AP_MAX_REGIONS) != cudaSuccess ||
+        cudaMemset(c->stats, 0, sizeof(ap::dev_stats) * ap::STAT_SHARDS) != cudaSuccess)
+        return fail(AP_ECUDA);
+    k_iota<<<c->num_sms, 256>>>(c->free_ids, frames);
+    if (cudaGetLastError() != cudaSuccess) return fail(AP_ECUDA);
+    c->h.pool = c->pool;
+    c->h.owner = c->owner;
+    c->h.free_ids = c->free_ids;
+    c->h.free_head = c->free_head;
+    c->h.clock_hand = c->clock_hand;
+    c->h.regions = c->regions;
+    c->h.stats = c->stats;
+    c->h.err = c->err;
+    c->h.frames = frames;
+    c->h.nfree = frames;
+    c->h.policy_seed = 0;
+    c->h.timeout_ns = 20000ull * 1000000ull;
+    c->h.log2_page = c->log2_page;
+    c->h.policy = ap::POLICY_CLOCK;
+    c->h.max_claims = 1;
+    c->h.sweep_steps = 64;
+    if (push_descriptor(c) != AP_OK) return fail(AP_ECUDA);
+    if (cudaDeviceSynchronize() != cudaSuccess) return fail(AP_ECUDA);
+    *out = c;
+    return AP_OK;
+}
+
+extern "C" int ap_cache_destroy(ap_cache_t c) {
+    if (!c) return AP_EINVAL;
+    for (auto& r : c->reg)
+        if (r.live) return AP_EBUSY;
+    ap_device_guard g(c->device);
+    cudaDeviceSynchronize();
+    cudaFree(c->pool_raw);
+    cudaFree(c->owner);
+    cudaFree(c->free_ids);
+    cudaFree(c->free_head);
+    cudaFree(c->regions);
+    cudaFree(c->stats);
+    cudaFree(c->d_cache);
+    delete c;
+    return AP_OK;
+}
+
+/* ------------------------------------------------------------ regions */
+extern "C" int ap_mmap(ap_cache_t c, const void* host_buf, uint64_t bytes, ap_region_t* out) {
+    if (!c || !host_buf || bytes == 0 || !out) return AP_EINVAL;
+    if (((uintptr_t)host_buf) & 15) return AP_EINVAL;
+    const uint64_t npages = (bytes + c->page - 1) >> c->log2_page;
+    if (npages >= (1ull << 48) || bytes >= (1ull << 60)) return AP_ERANGE;
+    uint32_t id = 0;
+    while (id < c->reg.size() && c->reg[id].live) ++id;
+    if (id >= AP_MAX_REGIONS) return AP_ERANGE;
+    ap_device_guard g(c->device);
+    ap_region_host rg;
+    rg.host_buf = host_buf;
+    rg.bytes = bytes;
+    rg.npages = npages;
+    cudaPointerAttributes attr{};
+    cudaError_t e = cudaPointerGetAttributes(&attr, host_buf);
+    cudaGetLastError();
+    if (e == cudaSuccess && attr.type == cudaMemoryTypeHost && attr.devicePointer) {
+        rg.dev_alias = (const uint8_t*)attr.devicePointer;
+    } else if (e == cudaSuccess && attr.type == cudaMemoryTypeDevice) {
+        return AP_EINVAL; /* the backing store is host memory */
+    } else {
+        unsigned flags = cudaHostRegisterMapped | cudaHostRegisterPortable;
+        int ro = 0;
+        cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->device);
+        if (ro) flags |= cudaHostRegisterReadOnly;
+        e = cudaHostRegister(const_cast<void*>(host_buf), bytes, flags);
+        if (e != cudaSuccess && ro) {
+            cudaGetLastError();
+            e = cudaHostRegister(const_cast<void*>(host_buf), bytes,
+                                 cudaHostRegisterMapped | cudaHostRegisterPortable);
+        }
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return AP_ENOMEM;
+        }
+        rg.registered = true;
+        void* dp = nullptr;
+        if (cudaHostGetDevicePointer(&dp, const_cast<void*>(host_buf), 0) != cudaSuccess) {
+            cudaHostUnregister(const_cast<void*>(host_buf));
+            return AP_ECUDA;
+        }
+        rg.dev_alias = (const uint8_t*)dp;
+    }
+    if (cudaMalloc(&rg.pte, npages * 8) != cudaSuccess) {
+        if (rg.registered) cudaHostUnregister(const_cast<void*>(host_buf));
+        cudaGetLastError();
+        return AP_ENOMEM;
+    }
+    AP_CUDA_TRY(cudaMemset(rg.pte, 0, npages * 8));
+    ap::dev_region d{};
+    d.host = rg.dev_alias;
+    d.bytes = bytes;
+    d.npages = npages;
+    d.pte = rg.pte;
+    d.cache = c->d_cache;
+    d.id = id;
+    d.live = 1;
+    AP_CUDA_TRY(cudaMemcpy(c->regions + id, &d, sizeof d, cudaMemcpyHostToDevice));
+    rg.live = true;
+    if (id == c->reg.size()) c->reg.push_back(rg);
+    else c->reg[id] = rg;
+    *out = id;
+    return AP_OK;
+}
+
+extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
+    if (!ap_region_ok(c, r)) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    ap_region_host& rg = c->reg[r];
+    int flag = 0;
+    int rc = scan_refs(c, rg, &flag);
+    if (rc) return rc;
+    if (flag) return AP_EBUSY;
+    k_drop_owner<<<c->num_sms * 4, 256>>>(c->owner, c->frames, (uint64_t)r + 1);
+    AP_CUDA_TRY(cudaGetLastError());
+    rc = rebuild_free_list(c);
+    if (rc) return rc;
+    AP_CUDA_TRY(cudaMemset(c->regions + r, 0, sizeof(ap::dev_region)));
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    cudaFree(rg.pte);
+    if (rg.registered) cudaHostUnregister(const_cast<void*>(rg.host_buf));
+    rg = ap_region_host{};
+    return AP_OK;
+}
+
+extern "C" int ap_region_devptr(ap_cache_t c, ap_region_t r, const void** out) {
+    if (!ap_region_ok(c, r) || !out) return AP_EINVAL;
+    *out = c->reg[r].dev_alias;
+    return AP_OK;
+}
+
+extern "C" int ap_region_npages(ap_cache_t c, ap_region_t r, uint64_t* npages) {
+    if (!ap_region_ok(c, r) || !npages) return AP_EINVAL;
+    *npages = c->reg[r].npages;
+    return AP_OK;
+}
+
+/* ------------------------------------------------------------ stats etc. */
+extern "C" int ap_cache_stats(ap_cache_t c, ap_stats_t* out) {
+    if (!c || !out) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    std::vector<ap::dev_stats> s(ap::STAT_SHARDS);
+    AP_CUDA_TRY(cudaMemcpy(s.data(), c->stats, sizeof(ap::dev_stats) * ap::STAT_SHARDS,
+                           cudaMemcpyDeviceToHost));
+    ap_stats_t t{};
+    for (auto& x : s) {
+        t.major += x.major;
+        t.minor += x.minor;
+        t.fill_bytes += x.fill_bytes;
+        t.evictions += x.evictions;
+        t.waits += x.waits;
+        t.downgrades += x.downgrades;
+        t.nofree += x.nofree;
+        t.unlinks += x.unlinks;
+    }
+    *out = t;
+    return AP_OK;
+}
+
+extern "C" int ap_cache_reset(ap_cache_t c) {
+    if (!c) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    for (auto& rg : c->reg) {
+        if (!rg.live) continue;
+        int flag = 0;
+        int rc = scan_refs(c, rg, &flag);
+        if (rc) return rc;
+        if (flag) return AP_EBUSY;
+    }
+    for (auto& rg : c->reg)
+        if (rg.live) AP_CUDA_TRY(cudaMemset(rg.pte, 0, rg.npages * 8));
+    AP_CUDA_TRY(cudaMemset(c->owner, 0, c->frames * 8));
+    AP_CUDA_TRY(cudaMemset(c->free_head, 0, 256));
+    AP_CUDA_TRY(cudaMemset(c->stats, 0, sizeof(ap::dev_stats) * ap::STAT_SHARDS));
+    k_iota<<<c->num_sms, 256>>>(c->free_ids, c->frames);
+    AP_CUDA_TRY(cudaGetLastError());
+    c->h.nfree = c->frames;
+    int rc = push_descriptor(c);
+    if (rc) return rc;
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    return AP_OK;
+}
+
+extern "C" int ap_cache_set_policy(ap_cache_t c, int policy, uint64_t seed) {
+    if (!c || (policy != AP_POLICY_CLOCK && policy != AP_POLICY_RANDOM)) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    c->h.policy = policy;
+    c->h.policy_seed = seed;
+    return push_descriptor(c);
+}
+
+extern "C" int ap_cache_set_tuning(ap_cache_t c, uint32_t max_claims, uint32_t sweep_steps,
+                                   uint32_t timeout_ms) {
+    if (!c || max_claims == 0 || max_claims > 32 || sweep_steps == 0) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    c->h.max_claims = max_claims;
+    c->h.sweep_steps = sweep_steps;
+    c->h.timeout_ns = (uint64_t)(timeout_ms ? timeout_ms : 20000) * 1000000ull;
+    return push_descriptor(c);
+}
+
+extern "C" int ap_last_device_error(ap_cache_t c) {
+    if (!c) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    int e = 0;
+    AP_CUDA_TRY(cudaMemcpy(&e, c->err, sizeof(int), cudaMemcpyDeviceToHost));
+    AP_CUDA_TRY(cudaMemset(c->err, 0, sizeof(int)));
+    return e;
+}
+
+extern "C" int ap_cache_dump(ap_cache_t c, uint64_t* owner_host, uint64_t* free_left) {
+    if (!c || !owner_host || !free_left) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    AP_CUDA_TRY(cudaMemcpy(owner_host, c->owner, c->frames * 8, cudaMemcpyDeviceToHost));
+    unsigned long long head = 0;
+    AP_CUDA_TRY(cudaMemcpy(&head, c->free_head, 8, cudaMemcpyDeviceToHost));
+    *free_left = head >= c->h.nfree ? 0 : c->h.nfree - head;
+    return AP_OK;
+}
+
+extern "C" int ap_region_dump_pte(ap_cache_t c, ap_region_t r, uint64_t* pte_host) {
+    if (!ap_region_ok(c, r) || !pte_host) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    AP_CUDA_TRY(cudaMemcpy(pte_host, c->reg[r].pte, c->reg[r].npages * 8, cudaMemcpyDeviceToHost));
+    return AP_OK;
+}
+
+extern "C" int ap_prefill(ap_cache_t c, ap_region_t r, uint64_t first, uint64_t npages,
+                          void* stream) {
+    if (!ap_region_ok(c, r) || first + npages > c->reg[r].npages) return AP_EINVAL;
+    if (npages == 0) return AP_OK;
+    ap_device_guard g(c->device);
+    const uint64_t warps = std::min<uint64_t>(npages, (uint64_t)c->num_sms * 32);
+    const unsigned blocks = (unsigned)((warps * 32 + 255) / 256);
+    k_prefill<<<blocks, 256, 0, (cudaStream_t)stream>>>(c->d_cache, r, first, npages);
+    AP_CUDA_TRY(cudaGetLastError());
+    return AP_OK;
+}

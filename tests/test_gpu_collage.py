@@ -1,0 +1,114 @@
+"""Parity of the collage kernel and the GPU-built LSH index against the oracle
+(O3): bucket CSR bit-exact, winners (image index, squared
+distance) bit-exact, for every candidate grouping, with the page cache smaller
+than the dataset (eviction) and on the raw-pointer twin."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from helpers import check_invariants, make_records
+
+pytestmark = pytest.mark.gpu
+
+
+def _setup(n, W, H, L, K, w, bb, seed=21, stride=4096, frames=256, page=4096):
+    recs = make_records(n, stride, seed)
+    proj, bias = synth.make_lsh_params(L, K, w, seed=seed + 1)
+    img, src, is_copy = synth.make_target(W, H, n, ds_seed=seed, seed=seed + 2, pool=32,
+                                          copy_permille=100)
+    return recs, proj, bias, img, src, is_copy
+
+
+def _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev):
+    L, K = bias.shape
+    off = torch.zeros((L, (1 << bb) + 1), dtype=torch.int32, device=dev)
+    ids = torch.zeros((L, n), dtype=torch.int32, device=dev)
+    pd = torch.from_numpy(proj).to(dev)
+    bd = torch.from_numpy(bias).to(dev)
+    ap.ap_lsh_build_index(cache, r, n, stride, L, K, bb, w, pd, bd, off, ids)
+    return off, ids, pd, bd
+
+
+@pytest.mark.parametrize("K,bb", [(8, 10), (0, 4), (3, 6)])
+def test_index_matches_oracle(ap, K, bb):
+    dev = torch.device("cuda:0")
+    n, stride, w = 3000, 4096, 2500
+    recs, proj, bias, *_ = _setup(n, 64, 64, 4, K, w, bb)
+    cache = ap.ap_cache_create(64, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, _, _ = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        want_off, want_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        assert np.array_equal(off.cpu().numpy().view(np.uint32), want_off)
+        assert np.array_equal(ids.cpu().numpy().view(np.uint32), want_ids)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("group", [1, 2, 4])
+@pytest.mark.parametrize("frames", [48, 5000])
+def test_collage_matches_oracle(ap, group, frames):
+    dev = torch.device("cuda:0")
+    n, stride, w, bb, L, K = 4096, 4096, 2500, 9, 4, 6
+    W, H = 512, 256
+    recs, proj, bias, img, src, is_copy = _setup(n, W, H, L, K, w, bb)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        inp = ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride, group=group)
+        ap.ap_collage_run(cache, r, inp, win)
+        torch.cuda.synchronize()
+        assert ap.ap_last_device_error(cache) == 0
+        got = win.cpu().numpy().view(np.uint32)
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n,
+                              off.cpu().numpy().view(np.uint32), ids.cpu().numpy().view(np.uint32))
+        assert np.array_equal(got, want)
+        # planted copies found at distance 0
+        assert np.all(got[is_copy.astype(bool), 1] == 0)
+        assert check_invariants(ap, cache, [r], frames) == []
+        # raw twin on a resident HBM copy of the file
+        rawd = torch.from_numpy(recs).to(dev)
+        win2 = torch.zeros_like(win)
+        inp2 = ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride, group=group,
+                             mode=ap.AP_MODE_RAW, raw_base=rawd)
+        ap.ap_collage_run(cache, r, inp2, win2)
+        torch.cuda.synchronize()
+        assert np.array_equal(win2.cpu().numpy().view(np.uint32), want)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+def test_collage_partitioned_blocks_equal_whole(ap):
+    """The multi-GPU partition on one GPU: block ranges run one
+    after the other and concatenated equal the single run."""
+    dev = torch.device("cuda:0")
+    n, stride, w, bb = 2048, 4096, 2500, 8
+    W, H = 256, 256
+    recs, proj, bias, img, *_ = _setup(n, W, H, 2, 5, w, bb, seed=5)
+    cache = ap.ap_cache_create(100, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        full = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n), full)
+        parts = []
+        for g in range(3):
+            b0, b1 = g * nb // 3, (g + 1) * nb // 3
+            part = torch.zeros((b1 - b0, 2), dtype=torch.int32, device=dev)
+            ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                      block_begin=b0, block_count=b1 - b0), part)
+            parts.append(part)
+        assert torch.equal(torch.cat(parts), full)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)

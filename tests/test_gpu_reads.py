@@ -1,0 +1,194 @@
+"""Parity of apointer reads (CUDA path through the C ABI) against the oracle
+(O1: plain file indexing) and the page-cache invariants (O2), across cache
+sizes, eviction policies, patterns and element sizes.  Every value must be
+bit-exact: faults and eviction order are invisible to values (PAPER.md:121,
+141-145)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from helpers import check_invariants, make_file
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture
+def dev():
+    assert torch.cuda.is_available(), "GPU tests need a B200"
+    return torch.device("cuda:0")
+
+
+def _run(ap, cache, region, cfg, nthreads, dev, out_bytes=None):
+    out = torch.zeros(out_bytes if out_bytes else nthreads * 8, dtype=torch.uint8, device=dev)
+    ap.ap_bench_read(cache, region, cfg, out)
+    torch.cuda.synchronize()
+    assert ap.ap_last_device_error(cache) == 0
+    return out.cpu().numpy()
+
+
+@pytest.mark.parametrize("frames", [1, 8, 64, 4096])
+@pytest.mark.parametrize("elem", [4, 16])
+def test_seq_copy_is_the_file(ap, dev, frames, elem):
+    """C1 shape: warps walk pages, every read faults while frames < pages."""
+    nbytes = (1 << 20) + 3 * 4096 + 48  # ragged last page
+    f = make_file(nbytes, seed=1)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        r = ap.ap_mmap(cache, f)
+        grid, block = (2, 64) if frames == 1 else (8, 128)
+        cfg = ap.bench_cfg(ap.AP_SEQ, elem, grid, block, unit_bytes=4096, out_copy=True,
+                           span_bytes=nbytes)
+        out = _run(ap, cache, r, cfg, grid * block, dev, out_bytes=nbytes)
+        whole = nbytes // elem * elem
+        assert np.array_equal(out[:whole], f[:whole])
+        assert check_invariants(ap, cache, [r], frames) == []
+        st = ap.ap_cache_stats(cache)
+        npages = (nbytes + 4095) // 4096
+        if frames >= npages:
+            assert st["major"] == npages and st["evictions"] == 0
+        else:
+            assert st["major"] >= npages and st["evictions"] >= npages - frames
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("elem,unit,passes", [(16, 4096, 1), (16, 16384, 3), (4, 2048, 2),
+                                              (8, 65536, 1)])
+def test_seq_checksums(ap, dev, elem, unit, passes):
+    page = 65536
+    nbytes = 4 * (1 << 20) + 777 * 16
+    f = make_file(nbytes, seed=2)
+    cache = ap.ap_cache_create(32, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        grid, block = 6, 256
+        cfg = ap.bench_cfg(ap.AP_SEQ, elem, grid, block, unit_bytes=unit, passes=passes,
+                           span_bytes=nbytes)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_seq(f, nbytes, unit, elem, grid * block, passes)
+        assert np.array_equal(got, want)
+        assert check_invariants(ap, cache, [r], 32) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("policy,seed", [(0, 0), (1, 1), (1, 2), (1, 3)])
+@pytest.mark.parametrize("frames", [3, 64, 2048])
+def test_uniform_random_any_eviction_order(ap, dev, policy, seed, frames):
+    page, nbytes = 4096, 4 << 20
+    f = make_file(nbytes, seed=3)
+    cache = ap.ap_cache_create(frames, page)
+    try:
+        ap.ap_cache_set_policy(cache, policy, seed)
+        r = ap.ap_mmap(cache, f)
+        grid, block, reads = 12, 128, 6
+        cfg = ap.bench_cfg(ap.AP_UNIFORM, 4, grid, block, reads_per_thread=reads, seed=99)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_uniform(f, nbytes, 4, grid * block, reads, 99)
+        assert np.array_equal(got, want)
+        assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("elem,page,frames", [(4, 4096, 256), (16, 4096, 40), (4, 65536, 64)])
+def test_divergent_distinct_pages(ap, dev, elem, page, frames):
+    nbytes = 200 * page
+    f = make_file(nbytes, seed=4)
+    cache = ap.ap_cache_create(frames, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        grid, block, reads = 8, 256, 4
+        cfg = ap.bench_cfg(ap.AP_DIVERGENT, elem, grid, block, reads_per_thread=reads,
+                           page_bytes=page, seed=5)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_divergent(f, nbytes, page, elem, grid * block, reads, 5)
+        assert np.array_equal(got, want)
+        assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+def test_hit_mode_after_prefill_has_no_major_faults(ap, dev):
+    page, nbytes, frames = 65536, 64 << 20, 1024
+    f = make_file(nbytes, seed=6)
+    cache = ap.ap_cache_create(frames, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        ap.ap_prefill(cache, r, 0, nbytes // page)
+        torch.cuda.synchronize()
+        st0 = ap.ap_cache_stats(cache)
+        assert st0["major"] == nbytes // page
+        grid, block = 148, 512
+        cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=16384, passes=2)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_seq(f, nbytes, 16384, 16, grid * block, 2)
+        assert np.array_equal(got, want)
+        st1 = ap.ap_cache_stats(cache)
+        assert st1["major"] == st0["major"]
+        # one link per (warp, unit) visit: SEQ with unit | page, all lanes on one page
+        assert st1["minor"] - st0["minor"] == 2 * (nbytes // 16384)
+        assert check_invariants(ap, cache, [r], frames) == []
+        # raw twin over an HBM copy reads the same values
+        dcopy = torch.from_numpy(f).to(dev)
+        cfg_raw = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=16384, passes=2,
+                               mode=ap.AP_MODE_RAW, raw_base=dcopy.data_ptr())
+        raw = _run(ap, cache, r, cfg_raw, grid * block, dev).view(np.uint64)
+        assert np.array_equal(raw, want)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+def test_zero_copy_raw_twin_uniform(ap, dev):
+    nbytes = 8 << 20
+    f = make_file(nbytes, seed=7)
+    cache = ap.ap_cache_create(16, 65536)
+    try:
+        r = ap.ap_mmap(cache, f)
+        base = ap.ap_region_devptr(cache, r)
+        cfg = ap.bench_cfg(ap.AP_UNIFORM, 4, 16, 256, reads_per_thread=3, seed=11,
+                           mode=ap.AP_MODE_RAW, raw_base=base)
+        got = _run(ap, cache, r, cfg, 16 * 256, dev).view(np.uint64)
+        assert np.array_equal(got, oracle.read_uniform(f, nbytes, 4, 16 * 256, 3, 11))
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+def test_two_regions_share_one_cache(ap, dev):
+    f1, f2 = make_file(3 << 20, seed=8), make_file(5 << 20, seed=9)
+    cache = ap.ap_cache_create(50, 4096)
+    try:
+        r1, r2 = ap.ap_mmap(cache, f1), ap.ap_mmap(cache, f2)
+        for r, f in ((r1, f1), (r2, f2), (r1, f1)):
+            cfg = ap.bench_cfg(ap.AP_UNIFORM, 4, 4, 256, reads_per_thread=4, seed=3)
+            got = _run(ap, cache, r, cfg, 1024, dev).view(np.uint64)
+            assert np.array_equal(got, oracle.read_uniform(f, f.nbytes, 4, 1024, 4, 3))
+        assert check_invariants(ap, cache, [r1, r2], 50) == []
+        ap.ap_munmap(cache, r1)
+        assert check_invariants(ap, cache, [r2], 50) == []
+        ap.ap_munmap(cache, r2)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+def test_reset_starts_cold(ap, dev):
+    f = make_file(2 << 20, seed=10)
+    cache = ap.ap_cache_create(600, 4096)
+    try:
+        r = ap.ap_mmap(cache, f)
+        cfg = ap.bench_cfg(ap.AP_SEQ, 16, 4, 128, unit_bytes=4096)
+        for _ in range(2):
+            ap.ap_cache_reset(cache)
+            _run(ap, cache, r, cfg, 512, dev)
+            st = ap.ap_cache_stats(cache)
+            assert st["major"] == 512 and st["evictions"] == 0
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
