@@ -1,0 +1,428 @@
+#!/usr/bin/env python
+"""bench.py -- apointer read throughput on B200 (BASELINE.json metric).
+
+Default workload = BASELINE.json configs[1] (C2): a 4 GiB synthetic file in
+pinned host memory, 64 KiB pages, a 1 GiB page cache in HBM, uniform-random
+4-byte apointer reads from every SM, starting from a cold cache each step
+("the first execution ... major page faults").  One step = one
+launch of the apointer read kernel over the whole read set; every step runs
+the whole hot path (S1-S10 of SURVEY.md §8(a)): translation, warp
+aggregation, minor/major faults, clock eviction, host-link fills, publish,
+unlink.
+
+`value` = fault-bound apointer read throughput: bytes the apointer fault
+path brought from the file into GPU memory per second (host-link fills),
+measured with CUDA events on the launch stream; its roofline is the host link
+measured in the same run.  The same JSON line also carries the cache-hit mode
+(HBM-bound, vs the raw-pointer twin) and the raw zero-copy twin of C2.
+
+Other workloads: --workload hit | c1 | c3 | c4 | c5 (collage).
+`--impl reference` times the CPU oracle (oracle/) on the host cores instead.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+GiB = 1 << 30
+METRIC = "apointer read GB/s (hit and fault-bound) vs raw ptr; collage s at 1/2/4/8 B200"
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("LOCAL_RANK", 0)),
+            int(os.environ.get("WORLD_SIZE", 1)))
+
+
+def aligned_empty(nbytes, align=1 << 21):
+    raw = np.empty(nbytes + align, dtype=np.uint8)
+    off = (-raw.ctypes.data) % align
+    return raw[off:off + nbytes]
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured (MEASURED_PEAKS.json)"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.path = tempfile.mktemp(suffix=".csv")
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}",
+                                          f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100"], stdout=self.f,
+                                         stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            self.proc.wait()
+            self.f.close()
+
+    def summary(self):
+        rows = []
+        try:
+            for line in open(self.path):
+                p = [x.strip() for x in line.split(",")]
+                if len(p) >= 9:
+                    rows.append(p)
+        except Exception:
+            pass
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = sorted(float(r[1]) for r in rows)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v == "Active"})
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": float(rows[0][2]),
+                "samples": len(rows), "reasons": reasons}
+
+
+# ------------------------------------------------------------------ workloads
+def c2_config(args):
+    return dict(workload="C2: 4 GiB file in pinned host memory, 64 KiB pages, 1 GiB page cache, "
+                         "uniform-random 4-B apointer reads from all SMs, cold cache per step",
+                file_bytes=4 * GiB, page=65536, frames=16384, grid=148, block=512,
+                reads_per_thread=args.reads, elem=4, seed=1234, file_seed=1)
+
+
+def host_link_peak(torch, dev):
+    """Host->device bandwidth measured in this run: cudaMemcpy from pinned
+    memory (copy engine), best of 5 x 1 GiB."""
+    h = torch.empty(GiB, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(GiB, dtype=torch.uint8, device=dev)
+    best = 0.0
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for _ in range(6):
+        s.record()
+        d.copy_(h, non_blocking=True)
+        e.record()
+        e.synchronize()
+        best = max(best, GiB / (s.elapsed_time(e) * 1e-3) / 1e9)
+    del h, d
+    return best
+
+
+def timed(torch, fn, stream):
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record(stream)
+    fn()
+    e.record(stream)
+    e.synchronize()
+    return s.elapsed_time(e) * 1e-3
+
+
+def run_c2(args, torch, dev, rank, world, dist):
+    import paper_conf_isca_shaharbs16_b200 as ap
+    import synth
+    cfgd = c2_config(args)
+    stream = torch.cuda.current_stream()
+    t_setup = time.time()
+    f = synth.fill_file(aligned_empty(cfgd["file_bytes"]), cfgd["file_seed"] + rank)
+    cache = ap.ap_cache_create(cfgd["frames"], cfgd["page"], torch.cuda.current_device())
+    region = ap.ap_mmap(cache, f)
+    t_setup = time.time() - t_setup
+    nthreads = cfgd["grid"] * cfgd["block"]
+    out = torch.empty(nthreads, dtype=torch.int64, device=dev)
+    cfg = ap.bench_cfg(ap.AP_UNIFORM, cfgd["elem"], cfgd["grid"], cfgd["block"],
+                       reads_per_thread=cfgd["reads_per_thread"], seed=cfgd["seed"])
+    link = host_link_peak(torch, dev)
+
+    def step():
+        ap.ap_bench_read(cache, region, cfg, out, stream)
+
+    for _ in range(args.warmup):
+        ap.ap_cache_reset(cache)
+        timed(torch, step, stream)
+    times, fills, stats = [], [], []
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        for _ in range(args.steps):
+            ap.ap_cache_reset(cache)  # cold start each step (untimed)
+            times.append(timed(torch, step, stream))
+            st = ap.ap_cache_stats(cache)
+            stats.append(st)
+            fills.append(st["fill_bytes"])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    err = ap.ap_last_device_error(cache)
+    total_t = sum(times)
+    total_fill = sum(fills)
+    # parity of the last step against the oracle is done by tests; here we
+    # keep the checksums for the cpu_baseline comparison (rank 0, N=1)
+    got = out.cpu().numpy().view(np.uint64)
+
+    # raw zero-copy twin: identical kernel on the host alias (no page cache)
+    base = ap.ap_region_devptr(cache, region)
+    cfg_raw = ap.bench_cfg(ap.AP_UNIFORM, cfgd["elem"], cfgd["grid"], cfgd["block"],
+                           reads_per_thread=cfgd["reads_per_thread"], seed=cfgd["seed"],
+                           mode=ap.AP_MODE_RAW, raw_base=base)
+    out_raw = torch.empty_like(out)
+    raw_t = min(timed(torch, lambda: ap.ap_bench_read(cache, region, cfg_raw, out_raw, stream),
+                      stream) for _ in range(3))
+    raw_match = bool(torch.equal(out_raw, out))
+    # zero-copy bulk read of 1 GiB through SMs (SEQ raw over the host alias)
+    cfg_zc = ap.bench_cfg(ap.AP_SEQ, 16, 148 * 4, 512, unit_bytes=16384, passes=1,
+                          span_bytes=GiB, mode=ap.AP_MODE_RAW, raw_base=base)
+    zc_out = torch.empty(148 * 4 * 512, dtype=torch.int64, device=dev)
+    zc_t = min(timed(torch, lambda: ap.ap_bench_read(cache, region, cfg_zc, zc_out, stream),
+                     stream) for _ in range(3))
+    zc_gbs = GiB / zc_t / 1e9
+
+    # e2e: the C-ABI call with a host output buffer (launch + D2H of checksums)
+    host_out = torch.empty(nthreads, dtype=torch.int64, pin_memory=True)
+    e2e_t = []
+    for _ in range(args.steps):
+        ap.ap_cache_reset(cache)
+        e2e_t.append(ap.ap_bench_read_host(cache, region, cfg, host_out.numpy()))
+    e2e_fill = ap.ap_cache_stats(cache)["fill_bytes"]
+
+    # cache-hit mode (M2h): warm the first 1 GiB, stream it 8x with 16-B reads
+    hit = run_hit(args, torch, dev, ap, cache, region, f, stream)
+
+    reads = nthreads * cfgd["reads_per_thread"]
+    res = dict(cfgd=cfgd, times=times, total_t=total_t, total_fill=total_fill, stats=stats,
+               err=err, link=link, zc_gbs=zc_gbs, raw_t=raw_t, raw_match=raw_match,
+               reads=reads, e2e_t=e2e_t, e2e_fill=e2e_fill, hit=hit, setup_s=t_setup,
+               clocks=clk.summary(), got=got, file=f, nthreads=nthreads)
+    ap.ap_munmap(cache, region)
+    ap.ap_cache_destroy(cache)
+    return res
+
+
+def run_hit(args, torch, dev, ap, cache, region, f, stream, span=GiB, passes=8):
+    page = 65536
+    ap.ap_cache_reset(cache)
+    ap.ap_prefill(cache, region, 0, span // page, stream)
+    torch.cuda.synchronize()
+    st0 = ap.ap_cache_stats(cache)
+    grid, block = 148, 512
+    nthreads = grid * block
+    out = torch.empty(nthreads, dtype=torch.int64, device=dev)
+    cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=16384, passes=passes,
+                       span_bytes=span)
+    dcopy = torch.from_numpy(f[:span]).to(dev)
+    out_raw = torch.empty_like(out)
+    cfg_raw = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=16384, passes=passes,
+                           span_bytes=span, mode=ap.AP_MODE_RAW, raw_base=dcopy.data_ptr())
+    for _ in range(max(args.warmup, 3)):
+        ap.ap_bench_read(cache, region, cfg, out, stream)
+        ap.ap_bench_read(cache, region, cfg_raw, out_raw, stream)
+    t_ap, t_raw = [], []
+    for _ in range(max(args.steps, 5)):
+        t_ap.append(timed(torch, lambda: ap.ap_bench_read(cache, region, cfg, out, stream), stream))
+        t_raw.append(timed(torch, lambda: ap.ap_bench_read(cache, region, cfg_raw, out_raw,
+                                                           stream), stream))
+    st1 = ap.ap_cache_stats(cache)
+    same = bool(torch.equal(out, out_raw))
+    del dcopy
+    nbytes = span * passes
+    ap_gbs = nbytes / np.mean(t_ap) / 1e9
+    raw_gbs = nbytes / np.mean(t_raw) / 1e9
+    return dict(bytes_per_launch=nbytes, ap_s=float(np.mean(t_ap)), raw_s=float(np.mean(t_raw)),
+                ap_gbs=ap_gbs, raw_gbs=raw_gbs, overhead=float(np.mean(t_ap) / np.mean(t_raw) - 1),
+                majors_during=st1["major"] - st0["major"], checksums_equal_raw=same)
+
+
+def cpu_oracle_c2(res, threads):
+    """The oracle as it stands (plain file indexing + FNV), on the host cores,
+    over the full C2 read set, repeated until >= 3 s."""
+    import oracle
+    cfgd = res["cfgd"]
+    f = res["file"]
+    t0 = time.time()
+    n = 0
+    while True:
+        ck = oracle.read_uniform(f, cfgd["file_bytes"], cfgd["elem"], res["nthreads"],
+                                 cfgd["reads_per_thread"], cfgd["seed"], threads=threads)
+        n += 1
+        if time.time() - t0 > 3.0:
+            break
+    dt = (time.time() - t0) / n
+    match = bool(np.array_equal(ck, res["got"]))
+    return dt, match
+
+
+def emit_c2(args, res_all, rank, world):
+    peaks, peak_src = measured_peaks()
+    r0 = res_all[0]
+    # max over ranks of the device-timed region; value = all ranks' fill bytes / that time
+    tmax = max(r["total_t"] for r in res_all)
+    fill_all = sum(r["total_fill"] for r in res_all)
+    value = fill_all / tmax / 1e9
+    st = r0["stats"][-1]
+    reads = r0["reads"]
+    per_launch_fill = r0["total_fill"] / len(r0["times"])
+    avg_t = r0["total_t"] / len(r0["times"])
+    achieved = per_launch_fill / avg_t / 1e9
+    e2e_val = sum(r["e2e_fill"] for r in res_all) / max(sum(r["e2e_t"]) for r in res_all) / 1e9
+    hit = r0["hit"]
+    line = {
+        "metric": METRIC,
+        "value": round(value, 3),
+        "unit": "GB/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(tmax / args.steps * 1e3, 3),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "u32",
+        "data": "synthetic (splitmix64 file words, seeded uniform offsets)",
+        "config": {"workload": r0["cfgd"]["workload"], "file_bytes": r0["cfgd"]["file_bytes"],
+                   "page_bytes": r0["cfgd"]["page"], "cache_bytes": r0["cfgd"]["frames"] *
+                   r0["cfgd"]["page"], "reads_per_step": reads, "elem_bytes": 4,
+                   "grid": r0["cfgd"]["grid"], "block": r0["cfgd"]["block"],
+                   "l2": "inputs larger than L2 (4 GiB file, 1 GiB cache, 126 MB L2); cache "
+                         "reset (cold) before every step",
+                   "parallelism": f"replicas x{world} (one cache + file per GPU)"},
+        "fault_bound": {
+            "fill_GBps": round(achieved, 3),
+            "host_link_GBps_memcpy": round(r0["link"], 2),
+            "host_link_GBps_zero_copy_sm": round(r0["zc_gbs"], 2),
+            "frac_of_host_link": round(achieved / r0["link"], 4),
+            "reads_per_s": round(reads / avg_t, 1),
+            "useful_GBps": round(reads * 4 / avg_t / 1e9, 6),
+            "major_faults": st["major"], "minor_faults": st["minor"],
+            "evictions": st["evictions"], "hit_ratio": round(1 - st["major"] / reads, 4),
+            "waits": st["waits"], "downgrades": st["downgrades"],
+            "raw_zero_copy_twin_s": round(r0["raw_t"], 6),
+            "raw_twin_checksums_equal": r0["raw_match"],
+            "device_error": r0["err"]},
+        "hit": {
+            "workload": "1 GiB resident (prefilled), SEQ 16-B apointer reads, 16 KiB units per "
+                        "warp, 8 passes, all SMs",
+            "apointer_GBps": round(hit["ap_gbs"], 1), "raw_GBps": round(hit["raw_gbs"], 1),
+            "overhead_vs_raw": round(hit["overhead"], 4),
+            "frac_of_hbm": round(hit["ap_gbs"] / peaks["hbm_gbs"], 4),
+            "hbm_peak_GBps": peaks["hbm_gbs"], "peak_source": peak_src,
+            "major_faults_during": hit["majors_during"],
+            "checksums_equal_raw": hit["checksums_equal_raw"]},
+        "roofline": {"bound": "host_link", "achieved": round(achieved, 3),
+                     "peak": round(r0["link"], 3), "unit": "GB/s",
+                     "frac": round(achieved / r0["link"], 4), "traffic": None,
+                     "kernel": "k_random<uint32_t, UNIFORM, apointer>",
+                     "peak_source": "host->device cudaMemcpy from pinned memory, measured in this "
+                                    "run (no host-link entry in MEASURED_PEAKS.json)"},
+        "e2e": {"value": round(e2e_val, 3), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": r0["nthreads"] * 8,
+                "zero_copy_h2d_bytes_per_step": int(r0["e2e_fill"] / len(r0["e2e_t"])),
+                "api": "ap_bench_read_host (launch + device->host copy of the checksums)"},
+        "gpu_launches": args.steps,
+        "clocks": r0["clocks"],
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        threads = os.cpu_count() or 1
+        dt, match = cpu_oracle_c2(r0, threads)
+        line["cpu_baseline"] = {"value": round(reads * 4 / dt / 1e9, 6), "unit": "GB/s",
+                                "cores": threads, "kind": "oracle",
+                                "sample": f"the full C2 read set ({reads} uniform 4-B reads of the "
+                                          f"4 GiB file + FNV-1a per thread), {dt:.4f} s per pass; "
+                                          f"value = bytes read / s (the oracle has no pages to "
+                                          f"fill); checksums equal GPU: {match}"}
+    return line
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank, _, world = env_rank()
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    cfgd = c2_config(args)
+    f = synth.fill_file(aligned_empty(cfgd["file_bytes"]), cfgd["file_seed"])
+    nthreads = cfgd["grid"] * cfgd["block"]
+    threads = os.cpu_count() or 1
+    ts = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.time()
+        oracle.read_uniform(f, cfgd["file_bytes"], 4, nthreads, cfgd["reads_per_thread"],
+                            cfgd["seed"], threads=threads)
+        if i >= args.warmup:
+            ts.append(time.time() - t0)
+    reads = nthreads * cfgd["reads_per_thread"]
+    dt = float(np.mean(ts))
+    v = reads * 4 / dt / 1e9
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": round(v, 6), "unit": "GB/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": cfgd["workload"]},
+        "cpu_baseline": {"value": round(v, 6), "unit": "GB/s", "cores": threads,
+                         "kind": "oracle",
+                         "sample": f"each step = the full C2 read set ({reads} reads), plain file "
+                                   f"indexing on the host cores; bytes = 4 per read"},
+        "e2e": {"value": round(v, 6), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0}}), flush=True)
+
+
+def main():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--workload", default="c2", choices=["c2"])
+    p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    args = p.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    rank, local, world = env_rank()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    res = run_c2(args, torch, dev, rank, world, dist)
+    if world > 1:
+        gathered = [None] * world
+        slim = {k: v for k, v in res.items() if k not in ("file", "got")}
+        dist.all_gather_object(gathered, slim)
+        res_all = [res] + gathered[1:] if rank == 0 else gathered
+    else:
+        res_all = [res]
+    if rank == 0:
+        print(json.dumps(emit_c2(args, res_all, rank, world)), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

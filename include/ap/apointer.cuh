@@ -261,7 +261,9 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         }
     }
     unsigned still = __ballot_sync(m, want && !got);
-    uint32_t steps = c->sweep_steps;
+    /* at most two laps of the clock per attempt (second chance), then back off */
+    const uint64_t lap = (c->frames + 31) / 32;
+    uint32_t steps = c->sweep_steps < 2 * lap + 1 ? c->sweep_steps : (uint32_t)(2 * lap + 1);
     unsigned long long evicted = 0;
     while (still && steps--) {
         unsigned long long hb = 0;
@@ -312,9 +314,11 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
  * S8 fill: the whole warp copies one page from pinned host memory (over the
  * host link, zero-copy 16-B loads) into frame `f`; a ragged last page is
  * zero-padded.  Host bytes are 16-B aligned (ap_mmap checks it). */
-__device__ __forceinline__ void fill_page(const dev_cache* c, const dev_region* r, uint64_t f,
-                                          uint64_t pg) {
-    const unsigned lane = lane_id();
+__device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, const dev_region* r,
+                                          uint64_t f, uint64_t pg) {
+    /* the lanes in m share the copy: rank = position among them */
+    const unsigned lane = __popc(m & lanemask_lt());
+    const unsigned nl = __popc(m);
     const uint64_t P = 1ull << c->log2_page;
     uint8_t* dst = c->pool + f * P;
     const uint8_t* src = r->host + pg * P;
@@ -325,17 +329,17 @@ __device__ __forceinline__ void fill_page(const dev_cache* c, const dev_region* 
     uint4* d4 = reinterpret_cast<uint4*>(dst);
     constexpr int U = 8;
     uint64_t i = lane;
-    for (; i + 32 * (U - 1) < nvec; i += 32 * U) {
+    for (; i + (uint64_t)nl * (U - 1) < nvec; i += (uint64_t)nl * U) {
         uint4 v[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) v[u] = __ldcs(s4 + i + 32 * u);
+        for (int u = 0; u < U; ++u) v[u] = __ldcs(s4 + i + (uint64_t)nl * u);
 #pragma unroll
-        for (int u = 0; u < U; ++u) __stcg(d4 + i + 32 * u, v[u]);
+        for (int u = 0; u < U; ++u) __stcg(d4 + i + (uint64_t)nl * u, v[u]);
     }
-    for (; i < nvec; i += 32) __stcg(d4 + i, __ldcs(s4 + i));
+    for (; i < nvec; i += nl) __stcg(d4 + i, __ldcs(s4 + i));
     if (len < P) {
         /* ragged tail: bytes [nvec*16, len) from host, the rest zeros */
-        for (uint64_t b = nvec * 16 + lane; b < P; b += 32)
+        for (uint64_t b = nvec * 16 + lane; b < P; b += nl)
             dst[b] = b < len ? src[b] : (uint8_t)0;
     }
 }
@@ -370,6 +374,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
     const uint64_t pg = need ? (x >> lg) : 0;
     const unsigned long long mykey = ((unsigned long long)r->id << 48) | pg;
     bool linked_here = false;
+    bool held = !need && (x >> 63); /* linked before this call: value already loaded */
     uint64_t t0 = 0;
     uint32_t backoff = 64;
     int idle_rounds = 0;
@@ -386,7 +391,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
 
         /* Phase A (leaders, lane-parallel; R-A13): minor faults link at once;
          * up to max_claims leaders (lane order) may claim an EMPTY entry. */
-        enum { ST_NONE = 0, ST_LINKED = 1, ST_CLAIMED = 2, ST_WAIT = 3, ST_SKIP = 4 };
+        enum { ST_NONE = 0, ST_LINKED = 1, ST_CLAIMED = 2, ST_WAIT = 3, ST_SKIP = 4, ST_NOFRAME = 5 };
         int st = ST_NONE;
         uint32_t frame = 0;
         uint64_t old = is_leader ? ld_acquire(pte) : 0;
@@ -429,7 +434,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame);
             if (st == ST_CLAIMED && !ok) {
                 st_release(pte, PTE_EMPTY); /* give the page back; retry later */
-                st = ST_WAIT;
+                st = ST_NOFRAME;
             }
         }
 
@@ -446,7 +451,11 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             const dev_region* fr =
                 reinterpret_cast<const dev_region*>(__shfl_sync(m, (unsigned long long)r, L));
             if ((int)lane == L) st_relaxed(c->owner + f, ((uint64_t)(fr->id + 1) << 48) | fpg);
-            fill_page(c, fr, f, fpg);
+            fill_page(m, c, fr, f, fpg);
+            if ((int)lane == __ffs(m) - 1) {
+                const uint64_t avail = fr->bytes - (fpg << lg);
+                stat_add(&S->fill_bytes, avail < P ? avail : P);
+            }
             fence_gpu();
             __syncwarp(m);
             if ((int)lane == L)
@@ -479,25 +488,31 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         if (waiting) {
             /* Under pressure (free list empty), stop pinning pages whose values
              * are already in registers (PAPER.md:115 heuristic; R-A19). */
+            /* With no frame to be had anywhere (or a long wait), also release
+             * lanes that came in linked: their values were loaded on entry.
+             * Then every waiting warp holds no pin for this pointer, so some
+             * warp can always allocate (deadlock freedom, R-A19). */
             const bool pressure = *(volatile unsigned long long*)c->free_head >= c->nfree;
             const bool waited = __any_sync(m, is_leader && st == ST_WAIT);
-            if (pressure || (waited && idle_rounds >= 2)) {
-                const bool dg = linked_here;
+            const bool hard = __any_sync(m, st == ST_NOFRAME) || (waited && idle_rounds >= 2);
+            if (pressure || hard) {
+                const bool dg = linked_here || (hard && held);
                 if (__any_sync(m, dg)) {
                     unlink_lanes(m, dg, r, page);
                     if (dg) {
                         x = (page << lg) | (x & (P - 1));
                         linked_here = false;
+                        held = false;
                     }
                     const unsigned ndg = __popc(__ballot_sync(m, dg));
                     if ((int)lane == __ffs(m) - 1) stat_add(&S->downgrades, ndg);
                 }
             }
+            if (t0 == 0) t0 = now_ns();
             if (!progressed) {
                 ++idle_rounds;
                 if ((int)lane == __ffs(m) - 1) stat_add(&S->waits, 1);
-                if (t0 == 0) t0 = now_ns();
-                else if (now_ns() - t0 > c->timeout_ns) {
+                if (now_ns() - t0 > c->timeout_ns) {
                     /* watchdog: give up on the remaining lanes (value 0). */
                     if (need) {
                         set_err(c, ERR_TIMEDOUT);
@@ -511,7 +526,6 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             } else {
                 idle_rounds = 0;
                 backoff = 64;
-                t0 = 0;
             }
         }
     }
