@@ -358,9 +358,12 @@ struct slow_out {
  * value at the lane's offset for lanes that were unlinked. */
 template <class T>
 __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t page,
-                                               const dev_region* r, T val_in) {
-    T vv = val_in;
-    T* val = &vv;
+                                               const dev_region* r) {
+    /* Lanes linked on entry reload their value here, so the caller's
+     * speculative load is dead on this path and is never kept live across
+     * the call (keeping it live made every hit-path load wait for its data
+     * before the vote's branch). */
+    T vv = (x >> 63) ? ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR)) : T{};
     const dev_cache* c = r->cache;
     const unsigned lane = lane_id();
     const uint32_t lg = c->log2_page;
@@ -368,7 +371,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
     bool need = !(x >> 63);
     if (need && (x + sizeof(T) > r->bytes || (x % sizeof(T)) != 0)) {
         set_err(c, ERR_FAULT);
-        *val = T{};
+        vv = T{};
         need = false;
     }
     const uint64_t pg = need ? (x >> lg) : 0;
@@ -473,7 +476,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             page = pg;
             need = false;
             linked_here = true;
-            *val = ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
+            vv = ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
             progressed = true;
         }
         if ((int)lane == __ffs(m) - 1) {
@@ -516,7 +519,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
                     /* watchdog: give up on the remaining lanes (value 0). */
                     if (need) {
                         set_err(c, ERR_TIMEDOUT);
-                        *val = T{};
+                        vv = T{};
                         need = false;
                     }
                     continue;
@@ -530,6 +533,29 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         }
     }
     return slow_out<T>{x, page, vv};
+}
+
+template <class T, int N>
+struct tile_out {
+    T v[N];
+};
+
+/* Element-wise tile read for tiles that straddle a page: each element goes
+ * through a temporary unlinked pointer (fault, read, unlink). */
+template <class T, int N>
+__device__ AP_SLOW_ATTR tile_out<T, N> read_tile_slow(unsigned m, uint64_t x, uint64_t page,
+                                                      const dev_region* r, uint32_t lg,
+                                                      int64_t stride) {
+    tile_out<T, N> t;
+    const uint64_t f0 = (x >> 63) ? ((page << lg) | (x & ((1ull << lg) - 1))) : x;
+    for (int k = 0; k < N; ++k) {
+        const uint64_t fk = f0 + (uint64_t)(k * stride * (int64_t)sizeof(T));
+        const slow_out<T> o = deref_slow<T>(m, fk, 0, r);
+        t.v[k] = o.val;
+        const bool l = (o.x >> 63) != 0;
+        if (__any_sync(m, l)) unlink_lanes(m, l, r, o.page);
+    }
+    return t;
 }
 
 }  // namespace detail
@@ -575,7 +601,7 @@ struct ptr {
         const T* a = v ? reinterpret_cast<const T*>(x & XL_ADDR) : reinterpret_cast<const T*>(r);
         T val = detail::ld_data<T>(a); /* speculative prefetch */
         if (__all_sync(m, v)) return val;
-        const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r, val);
+        const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
         x = o.x;
         page = o.page;
         return o.val;
@@ -594,6 +620,41 @@ struct ptr {
         ptr q(*this);
         q.x += nb;
         return *q;
+    }
+
+    /* Tiled read: v[k] = p[k * stride] for k < N, p unchanged.  One
+     * translation check covers the whole tile when every lane is linked and
+     * its tile stays inside its page; the N loads then issue back to back
+     * (memory tiling; one check per tile instead of per access
+     * is the hand-written form of the check elimination PAPER.md:450 asks of
+     * a compiler).  An unlinked pointer is first linked by dereferencing its
+     * first element (the usual fault path); a tile that straddles a page is
+     * read element by element.  No loaded value is ever live across a call
+     * into the fault path, so the tile stays in registers. */
+    template <int N>
+    __device__ __forceinline__ void read_tile(T (&v)[N], int64_t stride) {
+        const unsigned m = __activemask();
+        const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
+        bool ok = linked() && ((x ^ (x + span)) >> lg) == 0;
+        if (!__all_sync(m, ok)) {
+            if (__any_sync(m, !linked())) {
+                const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
+                x = o.x;
+                page = o.page;
+            }
+            ok = linked() && ((x ^ (x + span)) >> lg) == 0;
+            if (!__all_sync(m, ok)) {
+                /* hold no pin while the element-wise path faults (R-A19) */
+                release();
+                const detail::tile_out<T, N> t = detail::read_tile_slow<T, N>(m, x, page, r, lg, stride);
+#pragma unroll
+                for (int k = 0; k < N; ++k) v[k] = t.v[k];
+                return;
+            }
+        }
+        const T* a = reinterpret_cast<const T*>(x & XL_ADDR);
+#pragma unroll
+        for (int k = 0; k < N; ++k) v[k] = detail::ld_data<T>(a + k * stride);
     }
 
     /* S4: arithmetic.  Staying inside the page keeps the link; leaving it

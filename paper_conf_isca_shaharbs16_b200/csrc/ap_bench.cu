@@ -106,11 +106,8 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
                 if (whole) {
                     for (; j + TILE <= per_unit; j += TILE) {
                         T v[TILE];
-#pragma unroll
-                        for (int k = 0; k < TILE; ++k) {
-                            v[k] = *q;
-                            q += 32;
-                        }
+                        q.read_tile(v, 32);
+                        q += 32 * TILE;
 #pragma unroll
                         for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
                     }
