@@ -174,6 +174,37 @@ __device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+__device__ __forceinline__ uint64_t cas_acquire(uint64_t* p, uint64_t cmp, uint64_t val) {
+    uint64_t old;
+    asm volatile("atom.acquire.gpu.global.cas.b64 %0, [%1], %2, %3;"
+                 : "=l"(old) : "l"(p), "l"(cmp), "l"(val) : "memory");
+    return old;
+}
+__device__ __forceinline__ uint64_t cas_relaxed(uint64_t* p, uint64_t cmp, uint64_t val) {
+    uint64_t old;
+    asm volatile("atom.relaxed.gpu.global.cas.b64 %0, [%1], %2, %3;"
+                 : "=l"(old) : "l"(p), "l"(cmp), "l"(val) : "memory");
+    return old;
+}
+__device__ __forceinline__ uint64_t add_acquire(uint64_t* p, uint64_t v) {
+    uint64_t old;
+    asm volatile("atom.acquire.gpu.global.add.u64 %0, [%1], %2;"
+                 : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ void red_add_relaxed(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_or_relaxed(uint64_t* p, uint64_t v) {
+    asm volatile("red.relaxed.gpu.global.or.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long fetch_add_relaxed(unsigned long long* p,
+                                                                unsigned long long v) {
+    unsigned long long old;
+    asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;"
+                 : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
 
 __device__ __forceinline__ uint64_t sm64(uint64_t x) {
     uint64_t z = x + 0x9e3779b97f4a7c15ull;
@@ -208,7 +239,7 @@ __device__ __forceinline__ dev_stats* my_stats(const dev_cache* c) {
     return c->stats + (sm_id() % STAT_SHARDS);
 }
 __device__ __forceinline__ void stat_add(unsigned long long* ctr, unsigned long long v) {
-    if (v) atomicAdd(ctr, v);
+    if (v) red_add_relaxed(ctr, v);
 }
 
 /* k-th (0-based) set bit of m; m must have > k set bits. */
@@ -252,7 +283,7 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         unsigned long long base = ~0ull;
         if ((int)lane == first) {
             if (*(volatile unsigned long long*)c->free_head < c->nfree)
-                base = atomicAdd(c->free_head, (unsigned long long)k);
+                base = fetch_add_relaxed(c->free_head, (unsigned long long)k);
         }
         base = __shfl_sync(m, base, first);
         if (want && base != ~0ull && base + rank < c->nfree) {
@@ -268,7 +299,7 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
     while (still && steps--) {
         unsigned long long hb = 0;
         if ((int)lane == first)
-            hb = atomicAdd(c->clock_hand, c->policy == POLICY_CLOCK ? 32ull : 1ull);
+            hb = fetch_add_relaxed(c->clock_hand, c->policy == POLICY_CLOCK ? 32ull : 1ull);
         hb = __shfl_sync(m, hb, first);
         uint64_t f;
         if (c->policy == POLICY_CLOCK) f = (hb + lane) % c->frames;
@@ -282,14 +313,14 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
             q = vr->pte + (own & PAGE_MASK48);
             e = ld_relaxed(q);
             if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f && (e & PTE_RC_MASK) == 0) {
-                if (c->policy == POLICY_CLOCK && (e & PTE_REF)) cas_acq_rel(q, e, e & ~PTE_REF);
+                if (c->policy == POLICY_CLOCK && (e & PTE_REF)) cas_relaxed(q, e, e & ~PTE_REF);
                 else elig = true;
             }
         }
         const unsigned cand = __ballot_sync(m, elig);
         const int need_n = __popc(still);
         bool won = false;
-        if (elig && __popc(cand & lanemask_lt()) < need_n) won = (cas_acq_rel(q, e, PTE_EMPTY) == e);
+        if (elig && __popc(cand & lanemask_lt()) < need_n) won = (cas_acquire(q, e, PTE_EMPTY) == e);
         const unsigned wonm = __ballot_sync(m, won);
         const int nwon = __popc(wonm);
         evicted += nwon;
@@ -397,37 +428,37 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         enum { ST_NONE = 0, ST_LINKED = 1, ST_CLAIMED = 2, ST_WAIT = 3, ST_SKIP = 4, ST_NOFRAME = 5 };
         int st = ST_NONE;
         uint32_t frame = 0;
-        uint64_t old = is_leader ? ld_acquire(pte) : 0;
+        /* Optimistic link: one acquire add of n.  If the entry was VALID the
+         * group is linked (one round trip for a minor fault); otherwise the
+         * add is undone.  Every other transition tolerates such transient
+         * counts on non-VALID entries: publish and revert are adds, claims
+         * are CASes from exactly EMPTY (R-A17). */
+        uint64_t old = is_leader ? add_acquire(pte, n) : 0;
+        if (is_leader) {
+            if ((old >> 62) == 2) {
+                st = ST_LINKED;
+                frame = (uint32_t)((old >> 32) & PTE_FRAME_MASK);
+                if (!(old & PTE_REF)) red_or_relaxed(pte, PTE_REF);
+            } else {
+                red_add_relaxed(reinterpret_cast<unsigned long long*>(pte),
+                                (unsigned long long)(0 - (uint64_t)n));
+            }
+        }
         const unsigned empties = __ballot_sync(m, is_leader && (old >> 62) == 0);
         const bool may_claim = !((empties >> lane) & 1u) ||
                                (uint32_t)__popc(empties & lanemask_lt()) < c->max_claims;
-        if (is_leader) {
-            for (;;) {
-                const uint64_t s = old >> 62;
-                if (s == 2) {
-                    const uint64_t nw = (old + n) | PTE_REF;
-                    const uint64_t prev = cas_acq_rel(pte, old, nw);
-                    if (prev == old) {
-                        st = ST_LINKED;
-                        frame = (uint32_t)((old >> 32) & PTE_FRAME_MASK);
-                        break;
-                    }
-                    old = prev;
-                } else if (s == 0) {
-                    if (!may_claim) {
-                        st = ST_SKIP;
-                        break;
-                    }
-                    const uint64_t prev = cas_acq_rel(pte, old, PTE_LOADING);
-                    if (prev == old) {
-                        st = ST_CLAIMED;
-                        break;
-                    }
-                    old = prev;
+        if (is_leader && st == ST_NONE) {
+            if ((old >> 62) == 0) {
+                if (!may_claim) {
+                    st = ST_SKIP;
                 } else {
-                    st = ST_WAIT;
-                    break;
+                    const uint64_t prev = cas_acquire(pte, PTE_EMPTY, PTE_LOADING);
+                    /* prev != 0: transient counts, a racing claimer or a
+                     * publish in between; all resolve by retrying */
+                    st = prev == PTE_EMPTY ? ST_CLAIMED : ST_WAIT;
                 }
+            } else {
+                st = ST_WAIT; /* LOADING by another warp */
             }
         }
 
@@ -436,7 +467,8 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         if (claimed) {
             const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame);
             if (st == ST_CLAIMED && !ok) {
-                st_release(pte, PTE_EMPTY); /* give the page back; retry later */
+                /* give the page back (an add, so transient counts survive) */
+                red_add_release(pte, (uint64_t)0 - PTE_LOADING);
                 st = ST_NOFRAME;
             }
         }
@@ -462,7 +494,8 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             fence_gpu();
             __syncwarp(m);
             if ((int)lane == L)
-                st_release(pte, PTE_VALID | PTE_REF | ((uint64_t)f << 32) | (uint64_t)n);
+                red_add_release(pte, (PTE_VALID - PTE_LOADING) | PTE_REF | ((uint64_t)f << 32) |
+                                         (uint64_t)n);
         }
         const unsigned nminor = __popc(__ballot_sync(m, st == ST_LINKED));
 

@@ -7,7 +7,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libapointer.so")
+LIB_PATH = os.environ.get("AP_LIB_PATH") or os.path.join(_HERE, "libapointer.so")
 
 AP_OK = 0
 AP_EINVAL, AP_ENOMEM, AP_ECUDA, AP_EBUSY, AP_ERANGE = -1, -2, -3, -4, -5

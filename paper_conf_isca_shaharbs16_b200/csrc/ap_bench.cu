@@ -76,7 +76,10 @@ __device__ __forceinline__ uint64_t divergent_off(const BenchArgs& a, uint32_t E
 /* Loads are tiled TILE deep ("memory tiling ... interleaves
  * memory copy operations"): TILE dereferences are issued before the values
  * are consumed, so each warp keeps TILE requests in flight. */
-constexpr int TILE = 8;
+#ifndef AP_TILE
+#define AP_TILE 8
+#endif
+constexpr int TILE = AP_TILE;
 
 template <class T>
 __device__ __forceinline__ void consume(const BenchArgs& a, uint64_t off, const T& v,
@@ -107,9 +110,11 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
                     for (; j + TILE <= per_unit; j += TILE) {
                         T v[TILE];
                         q.read_tile(v, 32);
-                        q += 32 * TILE;
 #pragma unroll
                         for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
+                        /* advance after the values are used: a page-leaving
+                         * step then unlinks with no loads still in flight */
+                        q += 32 * TILE;
                     }
                 }
                 for (; j < per_unit; ++j) {

@@ -25,7 +25,8 @@ cache = ap.ap_cache_create(16384, 65536)
 r = ap.ap_mmap(cache, f)
 ap.ap_prefill(cache, r, 0, span // 65536)
 torch.cuda.synchronize()
-grid, block = 148, 512
+import os
+grid, block = int(os.environ.get("AP_GRID", 148)), int(os.environ.get("AP_BLOCK", 512))
 out = torch.empty(grid * block, dtype=torch.int64, device=dev)
 out2 = torch.empty_like(out)
 dcopy = torch.from_numpy(f[:span]).to(dev)
