@@ -48,6 +48,16 @@ def aligned_empty(nbytes, align=1 << 21):
     return raw[off:off + nbytes]
 
 
+def ncu_traffic(kernel):
+    """dram read+write bytes per launch of `kernel` from the committed ncu
+    capture (profiles/traffic.json), or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f)[kernel]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
 def measured_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -333,7 +343,9 @@ def emit_c2(args, res_all, rank, world):
             "checksums_equal_raw": hit["checksums_equal_raw"]},
         "roofline": {"bound": "host_link", "achieved": round(achieved, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
-                     "frac": round(achieved / r0["link"], 4), "traffic": None,
+                     "frac": round(achieved / r0["link"], 4),
+                     "traffic": ncu_traffic("k_random<uint32_t, UNIFORM, apointer>"),
+                     "algorithmic_bytes_per_launch": int(per_launch_fill),
                      "kernel": "k_random<uint32_t, UNIFORM, apointer>",
                      "peak_source": "host->device cudaMemcpy from pinned memory, measured in this "
                                     "run (no host-link entry in MEASURED_PEAKS.json)"},
@@ -399,7 +411,8 @@ def main():
     p.add_argument("--steps", type=int, default=5)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--workload", default="c2", choices=["c2"])
+    p.add_argument("--workload", default="c2", choices=["c2", "c4", "c5"])
+    p.add_argument("--group", type=int, default=1, help="collage candidates per warp")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     args = p.parse_args()
@@ -414,16 +427,27 @@ def main():
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=dev)
-    res = run_c2(args, torch, dev, rank, world, dist)
+    if args.workload in ("c4", "c5"):
+        import bench_collage
+        res = bench_collage.run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler,
+                                        host_link_peak)
+        drop = ("got", "is_copy", "src")
+    else:
+        res = run_c2(args, torch, dev, rank, world, dist)
+        drop = ("file", "got")
     if world > 1:
         gathered = [None] * world
-        slim = {k: v for k, v in res.items() if k not in ("file", "got")}
+        slim = {k: v for k, v in res.items() if k not in drop}
         dist.all_gather_object(gathered, slim)
         res_all = [res] + gathered[1:] if rank == 0 else gathered
     else:
         res_all = [res]
     if rank == 0:
-        print(json.dumps(emit_c2(args, res_all, rank, world)), flush=True)
+        if args.workload in ("c4", "c5"):
+            line = bench_collage.emit_collage(args, res_all, world, METRIC)
+        else:
+            line = emit_c2(args, res_all, rank, world)
+        print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()

@@ -1,0 +1,253 @@
+"""Collage workloads for bench.py (--workload c4 | c5): PAPER.md:405-442.
+
+C4 (BASELINE configs[3]): 1M 32x32 tiles (4 GiB file of 4 KiB-padded
+histograms), 1024x1024 target, LSH candidate lists, integer SSD, 1 B200.
+C5 (configs[4]): 10M tiles (40.96 GB pinned host file), 8192x8192 target,
+query blocks partitioned over the ranks, each with its own 2 GiB page cache,
+one NCCL gather of the per-block winners to rank 0.
+
+A step = reset the cache (cold, untimed), then the collage kernel over this
+rank's block range (+ the gather when N > 1), timed with CUDA events on the
+launch stream; the step time is the max over ranks.
+"""
+import json
+import mmap
+import os
+import time
+
+import numpy as np
+
+GiB = 1 << 30
+LSH_SEED, DS_SEED, TGT_SEED = 22, 21, 23
+
+
+def collage_config(name):
+    if name == "c4":
+        return dict(name="c4", N=1 << 20, W=1024, H=1024, L=4, K=8, bb=14, w=60000,
+                    frames=65536, page=4096, stride=4096,
+                    workload="C4: 1M 32x32 RGB tiles (4 GiB file of 4 KiB-padded histograms in "
+                             "pinned host memory), 1024x1024 target, LSH L=4 K=8 2^14 buckets, "
+                             "integer SSD, 256 MiB page cache (cold per step), 1 B200")
+    return dict(name="c5", N=10_000_000, W=8192, H=8192, L=4, K=8, bb=16, w=60000,
+                frames=524288, page=4096, stride=4096,
+                workload="C5: 10M tiles in a 40.96 GB pinned host file, 8192x8192 target, LSH "
+                         "L=4 K=8 2^16 buckets, query blocks partitioned over the ranks, 2 GiB "
+                         "page cache per GPU (cold per step), one NCCL gather of the winners")
+
+
+def _shm_records(cfg, rank, world, dist):
+    """The record file in /dev/shm, generated once (all ranks map the same
+    pages; each rank registers them for its own GPU)."""
+    import synth
+    nbytes = cfg["N"] * cfg["stride"]
+    path = f"/dev/shm/apb_{cfg['name']}_{cfg['N']}_{cfg['stride']}_{DS_SEED}.bin"
+    done = path + ".ok"
+    if rank == 0 and not os.path.exists(done):
+        with open(path, "wb") as fh:
+            fh.truncate(nbytes)
+        with open(path, "r+b") as fh:
+            mm = mmap.mmap(fh.fileno(), nbytes)
+            arr = np.frombuffer(mm, dtype=np.uint8)
+            chunk = 1 << 18
+            for first in range(0, cfg["N"], chunk):
+                cnt = min(chunk, cfg["N"] - first)
+                synth.fill_records(arr[first * cfg["stride"]:(first + cnt) * cfg["stride"]], first,
+                                   cnt, cfg["stride"], DS_SEED)
+            del arr
+            mm.flush()
+            mm.close()
+        open(done, "w").close()
+    if dist is not None:
+        dist.barrier()
+    fh = open(path, "r+b")
+    mm = mmap.mmap(fh.fileno(), nbytes)
+    return np.frombuffer(mm, dtype=np.uint8), (fh, mm)
+
+
+def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_link_peak):
+    import paper_conf_isca_shaharbs16_b200 as ap
+    import synth
+    cfg = collage_config(args.workload)
+    stream = torch.cuda.current_stream()
+    t0 = time.time()
+    if cfg["name"] == "c4":
+        from bench import aligned_empty
+        recs = synth.fill_records(aligned_empty(cfg["N"] * cfg["stride"]), 0, cfg["N"],
+                                  cfg["stride"], DS_SEED)
+        keep = None
+    else:
+        recs, keep = _shm_records(cfg, rank, world, dist)
+    img, src, is_copy = synth.make_target(cfg["W"], cfg["H"], cfg["N"], ds_seed=DS_SEED,
+                                          seed=TGT_SEED, pool=256, copy_permille=50)
+    proj, bias = synth.make_lsh_params(cfg["L"], cfg["K"], cfg["w"], seed=LSH_SEED)
+    t_gen = time.time() - t0
+    cache = ap.ap_cache_create(cfg["frames"], cfg["page"], torch.cuda.current_device())
+    t0 = time.time()
+    region = ap.ap_mmap(cache, recs)
+    t_pin = time.time() - t0
+    B = 1 << cfg["bb"]
+    off = torch.empty((cfg["L"], B + 1), dtype=torch.int32, device=dev)
+    ids = torch.empty((cfg["L"], cfg["N"]), dtype=torch.int32, device=dev)
+    pd, bd = torch.from_numpy(proj).to(dev), torch.from_numpy(bias).to(dev)
+    t0 = time.time()
+    ap.ap_lsh_build_index(cache, region, cfg["N"], cfg["stride"], cfg["L"], cfg["K"], cfg["bb"],
+                          cfg["w"], pd, bd, off, ids)
+    t_index = time.time() - t0
+    nb = (cfg["W"] // 32) * (cfg["H"] // 32)
+    b0, b1 = rank * nb // world, (rank + 1) * nb // world
+    tgt_host = torch.from_numpy(img).pin_memory()
+    tgt = tgt_host.to(dev)
+    win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
+    inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
+                        cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0)
+    gather_list = [torch.empty_like(win) for _ in range(world)] if (rank == 0 and world > 1) else None
+
+    def step():
+        ap.ap_collage_run(cache, region, inp, win, stream)
+        if world > 1:
+            dist.gather(win, gather_list, dst=0)
+
+    link = host_link_peak(torch, dev)
+    for _ in range(args.warmup):
+        ap.ap_cache_reset(cache)
+        if world > 1:
+            dist.barrier()
+        timed(torch, step, stream)
+    times, stats = [], []
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        for _ in range(args.steps):
+            ap.ap_cache_reset(cache)  # cold cache each step (untimed)
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            times.append(timed(torch, step, stream))
+            stats.append(ap.ap_cache_stats(cache))
+    err = ap.ap_last_device_error(cache)
+    got = win.cpu().numpy().view(np.uint32).copy()
+
+    # raw twin: identical kernel on a fully resident HBM copy (c4 only: 4 GiB)
+    raw = None
+    if cfg["name"] == "c4":
+        dcopy = torch.from_numpy(recs).to(dev)
+        inp_raw = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
+                                cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
+                                block_count=b1 - b0, mode=ap.AP_MODE_RAW, raw_base=dcopy)
+        win_raw = torch.empty_like(win)
+        for _ in range(2):
+            timed(torch, lambda: ap.ap_collage_run(cache, region, inp_raw, win_raw, stream), stream)
+        raw_t = min(timed(torch, lambda: ap.ap_collage_run(cache, region, inp_raw, win_raw, stream),
+                          stream) for _ in range(args.steps))
+        # apointer on the warm (fully resident would need 4 GiB of frames) cache:
+        # run the apointer kernel again without reset = warm-cache time
+        warm_t = min(timed(torch, lambda: ap.ap_collage_run(cache, region, inp, win, stream),
+                           stream) for _ in range(args.steps))
+        raw = dict(raw_s=raw_t, warm_s=warm_t, equal=bool(torch.equal(win_raw, win)))
+        del dcopy
+
+    # e2e through the public API: target H2D from pinned memory + kernel +
+    # winners D2H, per step, cold cache
+    host_win = torch.empty_like(win, device="cpu").pin_memory()
+    e2e = []
+    for _ in range(args.steps):
+        ap.ap_cache_reset(cache)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record(stream)
+        tgt.copy_(tgt_host, non_blocking=True)
+        ap.ap_collage_run(cache, region, inp, win, stream)
+        host_win.copy_(win, non_blocking=True)
+        e.record(stream)
+        e.synchronize()
+        e2e.append(s.elapsed_time(e) * 1e-3)
+    cands = None
+    res = dict(cfg=cfg, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
+               link=link, raw=raw, e2e=e2e, clocks=clk.summary(), t_gen=t_gen, t_pin=t_pin,
+               t_index=t_index, h2d=int(tgt_host.numel()), d2h=int(win.numel() * 4),
+               is_copy=is_copy, src=src, cands=cands)
+    # parity sample vs the oracle (rank 0): all blocks for c4, a sample for c5
+    res["parity"] = None
+    if rank == 0 and not args.no_cpu_baseline:
+        import oracle
+        o_off = off.cpu().numpy().view(np.uint32)
+        o_ids = ids.cpu().numpy().view(np.uint32)
+        threads = os.cpu_count() or 1
+        nsample = (b1 - b0) if cfg["name"] == "c4" else min(256, b1 - b0)
+        t0 = time.time()
+        want = oracle.collage(img, proj, bias, cfg["w"], cfg["bb"], recs, cfg["stride"], cfg["N"],
+                              o_off, o_ids, b0=b0, nb=nsample, threads=threads)
+        dt = time.time() - t0
+        res["parity"] = dict(blocks=nsample, equal=bool(np.array_equal(want, got[:nsample])),
+                             cpu_s=dt, cores=threads)
+        # the index itself vs the oracle's (c4: full; c5: skipped, 10M records)
+        if cfg["name"] == "c4":
+            po, pi = oracle.build_index(recs, cfg["stride"], cfg["N"], proj, bias, cfg["w"],
+                                        cfg["bb"], threads=threads)
+            res["parity"]["index_equal"] = bool(np.array_equal(po, o_off) and
+                                                np.array_equal(pi, o_ids))
+    ap.ap_munmap(cache, region)
+    ap.ap_cache_destroy(cache)
+    if keep:
+        del recs
+    return res
+
+
+def _traffic(kernel):
+    try:
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles",
+                               "traffic.json")) as f:
+            return json.load(f)[kernel]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
+def emit_collage(args, res_all, world, METRIC):
+    r0 = res_all[0]
+    cfg = r0["cfg"]
+    tmax = max(sum(r["times"]) for r in res_all) / args.steps
+    st = r0["stats"][-1]
+    fill = st["fill_bytes"]
+    t0 = sum(r0["times"]) / args.steps
+    line = {
+        "metric": METRIC, "value": round(tmax, 6), "unit": "s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tmax * 1e3, 3),
+        "higher_is_better": False, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic (blob-tile histograms, seeded target with 5% planted copies)",
+        "config": {"workload": cfg["workload"], "records": cfg["N"], "target": [cfg["W"], cfg["H"]],
+                   "blocks": r0["nb"], "L": cfg["L"], "K": cfg["K"], "bucket_bits": cfg["bb"],
+                   "w": cfg["w"], "cache_bytes_per_gpu": cfg["frames"] * cfg["page"],
+                   "group": args.group,
+                   "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",
+                   "parallelism": f"blocks partitioned over {world} rank(s) + NCCL gather"},
+        "collage": {"blocks_rank0": r0["b1"] - r0["b0"], "major_faults": st["major"],
+                    "minor_faults": st["minor"], "evictions": st["evictions"],
+                    "fill_GB": round(fill / 1e9, 3), "waits": st["waits"],
+                    "device_error": r0["err"], "setup_s": {"generate": round(r0["t_gen"], 2),
+                                                          "pin": round(r0["t_pin"], 2),
+                                                          "index_build_gpu": round(r0["t_index"], 3)},
+                    "per_rank_s": [round(sum(r["times"]) / args.steps, 6) for r in res_all]},
+        "roofline": {"bound": "host_link", "achieved": round(fill / t0 / 1e9, 3),
+                     "peak": round(r0["link"], 3), "unit": "GB/s",
+                     "frac": round(fill / t0 / 1e9 / r0["link"], 4),
+                     "traffic": _traffic(f"k_collage<{args.group}, apointer>"),
+                     "algorithmic_bytes_per_launch": int(fill),
+                     "kernel": f"k_collage<{args.group}, apointer>",
+                     "peak_source": "host->device cudaMemcpy from pinned memory, this run"},
+        "e2e": {"value": round(max(np.mean(r["e2e"]) for r in res_all), 6), "unit": "s",
+                "h2d_bytes_per_step": r0["h2d"], "d2h_bytes_per_step": r0["d2h"],
+                "api": "target H2D + ap_collage_run + winners D2H (cold cache)"},
+        "gpu_launches": args.steps,
+        "clocks": r0["clocks"],
+    }
+    if r0["raw"]:
+        line["collage"]["raw_twin_resident_hbm_s"] = round(r0["raw"]["raw_s"], 6)
+        line["collage"]["apointer_warm_cache_s"] = round(r0["raw"]["warm_s"], 6)
+        line["collage"]["overhead_warm_vs_raw"] = round(r0["raw"]["warm_s"] / r0["raw"]["raw_s"] - 1, 4)
+        line["collage"]["raw_twin_equal"] = r0["raw"]["equal"]
+    if r0["parity"]:
+        p = r0["parity"]
+        line["collage"]["parity_vs_oracle"] = {k: v for k, v in p.items() if k != "cpu_s"}
+        full_blocks = r0["b1"] - r0["b0"]
+        line["cpu_baseline"] = {"value": round(p["cpu_s"] * full_blocks / p["blocks"], 4),
+                                "unit": "s", "cores": p["cores"], "kind": "oracle",
+                                "sample": f"oracle collage over {p['blocks']} of rank 0's "
+                                          f"{full_blocks} blocks, scaled to all of them"}
+    return line

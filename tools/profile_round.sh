@@ -1,0 +1,19 @@
+#!/bin/bash
+# ncu evidence for profiles/: launch list of the default bench command, and
+# one --set full capture of each dominant kernel.  Run under gpurun (1 GPU).
+set -x
+mkdir -p gpurun_out
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+  --log-file gpurun_out/launches_c2.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline \
+  > gpurun_out/launches_c2.out 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_random -s 1 -c 1 \
+  -o gpurun_out/full_c2 python bench.py --steps 1 --warmup 1 --no-cpu-baseline \
+  > gpurun_out/full_c2.out 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_seq -c 1 \
+  -o gpurun_out/full_hit python tools/prof_hit.py 65536 2 > gpurun_out/full_hit.out 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_seq -s 6 -c 1 \
+  -o gpurun_out/full_hit_raw python tools/prof_hit.py 65536 2 > gpurun_out/full_hit_raw.out 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_collage -s 1 -c 1 \
+  -o gpurun_out/full_c4 python bench.py --workload c4 --steps 1 --warmup 1 --no-cpu-baseline \
+  > gpurun_out/full_c4.out 2>&1
+echo done
