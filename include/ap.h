@@ -164,7 +164,16 @@ typedef struct {
                                 * offsets (span bytes) instead of checksums      */
     const void* raw_base;      /* AP_MODE_RAW: device-readable file bytes (an HBM *
                                 * copy, or ap_region_devptr for zero-copy)       */
+    int32_t access;            /* SEQ, apointer mode: AP_ACCESS_TILE (default,    *
+                                * one translation check per 8 accesses),         *
+                                * AP_ACCESS_DEREF (`v = *q; q += 32` per access), *
+                                * AP_ACCESS_RANGE (one check per unit, then plain *
+                                * loads through the linked translation)          */
 } ap_bench_cfg;
+
+#define AP_ACCESS_TILE 0
+#define AP_ACCESS_DEREF 1
+#define AP_ACCESS_RANGE 2
 
 /* Run one microbenchmark launch (asynchronous on `stream`).
  * out_dev: uint64[grid*block] per-thread FNV-1a-64 checksums over the values

@@ -102,7 +102,8 @@ struct alignas(64) dev_region {
     const dev_cache* cache; /* owning cache                               */
     uint32_t id;            /* region id (< 65535)                        */
     uint32_t live;          /* 1 while mapped                             */
-    uint64_t pad_[2];
+    const uint8_t* pool;    /* the cache's frame pool (one hop for links) */
+    uint64_t pad_;
 };
 
 /* Cache descriptor, one copy in device memory per ap_cache_t. */
@@ -601,10 +602,10 @@ __device__ AP_SLOW_ATTR tile_out<T, N> read_tile_slow(unsigned m, uint64_t x, ui
 template <class T>
 struct ptr {
     static_assert(sizeof(T) == 4 || sizeof(T) == 8 || sizeof(T) == 16, "T must be 4/8/16 B");
-    uint64_t x;
-    const dev_region* r;
-    uint64_t page;
-    uint32_t lg;
+    uint64_t x;          /* translation field (R-A16)                       */
+    const dev_region* r; /* metadata: region                                */
+    uint64_t page;       /* metadata: linked page                           */
+    uint32_t lg;         /* metadata: log2(page size)                       */
 
     __device__ __forceinline__ ptr() : x(0), r(nullptr), page(0), lg(12) {}
     __device__ __forceinline__ ptr(const dev_region* reg, uint32_t log2_page, uint64_t foff)
@@ -617,6 +618,21 @@ struct ptr {
         x = nx;
         r = o.r;
         lg = o.lg;
+        return *this;
+    }
+    /* Move: the same pointer changes hands -- its link moves with it, no
+     * reference count changes. */
+    __device__ __forceinline__ ptr(ptr&& o) : x(o.x), r(o.r), page(o.page), lg(o.lg) {
+        o.detach();
+    }
+    __device__ __forceinline__ ptr& operator=(ptr&& o) {
+        if (this == &o) return *this;
+        release();
+        x = o.x;
+        r = o.r;
+        page = o.page;
+        lg = o.lg;
+        o.detach();
         return *this;
     }
     __device__ __forceinline__ ~ptr() { release(); }
@@ -690,6 +706,30 @@ struct ptr {
         for (int k = 0; k < N; ++k) v[k] = detail::ld_data<T>(a + k * stride);
     }
 
+    /* Translate once for a whole range: make the pointer linked and return
+     * its direct device address if [p, p + bytes) of every lane lies inside
+     * the page that lane links (else nullptr, nothing changed but a link).
+     * The address stays valid while this pointer stays linked -- a linked
+     * pointer keeps its page active and its mapping fixed (PAPER.md:113,
+     * 141) -- so a loop can stream through it with plain loads.  This is the
+     * per-page hoisting of the translation check that PAPER.md:450 expects
+     * from compiler support. */
+    __device__ __forceinline__ const T* pin_range(uint64_t bytes) {
+        const unsigned m = __activemask();
+        const uint64_t last = bytes ? bytes - 1 : 0;
+        bool ok = linked() && ((x ^ (x + last)) >> lg) == 0;
+        if (!__all_sync(m, ok)) {
+            if (__any_sync(m, !linked())) {
+                const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
+                x = o.x;
+                page = o.page;
+            }
+            ok = linked() && ((x ^ (x + last)) >> lg) == 0;
+            if (!__all_sync(m, ok)) return nullptr;
+        }
+        return reinterpret_cast<const T*>(x & XL_ADDR);
+    }
+
     /* S4: arithmetic.  Staying inside the page keeps the link; leaving it
      * unlinks with a warp-aggregated decrement (S10). */
     __device__ __forceinline__ ptr& operator+=(int64_t d) {
@@ -724,6 +764,10 @@ struct ptr {
             if (l) x = (page << lg) | (x & ((1ull << lg) - 1));
         }
     }
+
+   private:
+    /* Forget the link without touching the count (it moved elsewhere). */
+    __device__ __forceinline__ void detach() { x = foff(); }
 };
 
 /* gvmmap (M17): an unlinked apointer to byte offset

@@ -9,7 +9,7 @@ import ctypes
 import numpy as np
 
 from . import _lib
-from ._lib import (AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK,  # noqa: F401
+from ._lib import (AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_TILE, AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK,  # noqa: F401
                    AP_POLICY_RANDOM, AP_SEQ, AP_UNIFORM, APError, ap_bench_cfg, ap_collage_in,
                    ap_stats_t)
 
@@ -141,9 +141,9 @@ def ap_prefill(cache, region, first_page, npages, stream=None):
 
 def bench_cfg(pattern, elem_bytes, grid, block, reads_per_thread=0, passes=1, unit_bytes=0,
               page_bytes=0, span_bytes=0, seed=0, mode=AP_MODE_APOINTER, out_copy=False,
-              raw_base=None):
+              raw_base=None, access=AP_ACCESS_TILE):
     return ap_bench_cfg(pattern, elem_bytes, grid, block, reads_per_thread, passes, unit_bytes,
-                        page_bytes, span_bytes, seed, mode, int(out_copy), raw_base)
+                        page_bytes, span_bytes, seed, mode, int(out_copy), raw_base, access)
 
 
 def ap_bench_read(cache, region, cfg, out_dev, stream=None):

@@ -15,6 +15,7 @@ AP_EFAULT, AP_ENOFRAME, AP_ETIMEDOUT = -6, -7, -8
 AP_POLICY_CLOCK, AP_POLICY_RANDOM = 0, 1
 AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
+AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE = 0, 1, 2
 
 u64, u32, i32, vp, ci = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int
 
@@ -31,7 +32,7 @@ class ap_bench_cfg(ctypes.Structure):
     _fields_ = [("pattern", i32), ("elem_bytes", u32), ("grid", u32), ("block", u32),
                 ("reads_per_thread", u32), ("passes", u32), ("unit_bytes", u32),
                 ("page_bytes", u32), ("span_bytes", u64), ("seed", u64), ("mode", i32),
-                ("out_copy", i32), ("raw_base", vp)]
+                ("out_copy", i32), ("raw_base", vp), ("access", i32)]
 
 
 class ap_collage_in(ctypes.Structure):

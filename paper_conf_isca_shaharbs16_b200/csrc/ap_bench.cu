@@ -54,6 +54,7 @@ struct BenchArgs {
     uint64_t seed;
     const uint8_t* raw; /* RAW twin base                                */
     uint8_t* out_copy;  /* SEQ copy output or nullptr                   */
+    int32_t access;     /* AP_ACCESS_*                                  */
     uint64_t* ck;       /* per-thread checksums                         */
 };
 
@@ -73,11 +74,13 @@ __device__ __forceinline__ uint64_t divergent_off(const BenchArgs& a, uint32_t E
 }
 
 /* ------------------------------------------------------------ SEQ */
-/* Loads are tiled TILE deep ("memory tiling ... interleaves
- * memory copy operations"): TILE dereferences are issued before the values
- * are consumed, so each warp keeps TILE requests in flight. */
+/* Loads are tiled TILE deep and double-buffered ("memory
+ * tiling ... interleaves memory copy operations"): the next tile is issued
+ * before the current one is consumed, so each warp keeps up to 2*TILE 512-B
+ * requests in flight.  The apointer version and its raw twin run this same
+ * loop; only the reader differs. */
 #ifndef AP_TILE
-#define AP_TILE 8
+#define AP_TILE 16
 #endif
 constexpr int TILE = AP_TILE;
 
@@ -86,6 +89,56 @@ __device__ __forceinline__ void consume(const BenchArgs& a, uint64_t off, const 
                                         uint64_t& h) {
     if (a.out_copy) *reinterpret_cast<T*>(a.out_copy + off) = v;
     else h = fnv(h, v);
+}
+
+/* raw-pointer reader with the apointer's interface (the twin) */
+template <class T>
+struct raw_reader {
+    const T* p;
+    template <int N>
+    __device__ __forceinline__ void read_tile(T (&v)[N], int64_t stride) {
+#pragma unroll
+        for (int k = 0; k < N; ++k) v[k] = ap::detail::ld_data<T>(p + k * stride);
+    }
+    __device__ __forceinline__ raw_reader& operator+=(int64_t d) {
+        p += d;
+        return *this;
+    }
+    __device__ __forceinline__ T operator*() { return ap::detail::ld_data<T>(p); }
+};
+
+/* one unit, tiled: TILE loads issued before they are consumed */
+template <class T, class R>
+__device__ __forceinline__ void seq_unit(R& q, const BenchArgs& a, uint64_t e0, uint32_t per_unit,
+                                         bool whole, uint64_t& h) {
+    constexpr uint32_t E = sizeof(T);
+    uint32_t j = 0;
+    if (whole) {
+        for (; j + TILE <= per_unit; j += TILE) {
+            T v[TILE];
+            q.read_tile(v, 32);
+#pragma unroll
+            for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
+            q += 32 * TILE; /* after the values are used: no loads in flight at an unlink */
+        }
+    }
+    for (; j < per_unit; ++j) {
+        const uint64_t off = (e0 + 32ull * j) * E;
+        if (off + E <= a.span) consume(a, off, (T)*q, h);
+        q += 32;
+    }
+}
+
+/* one unit, one access at a time: `v = *q; q += 32` (the paper's loop) */
+template <class T>
+__device__ __forceinline__ void seq_unit_deref(ap::ptr<T>& q, const BenchArgs& a, uint64_t e0,
+                                               uint32_t per_unit, uint64_t& h) {
+    constexpr uint32_t E = sizeof(T);
+    for (uint32_t j = 0; j < per_unit; ++j) {
+        const uint64_t off = (e0 + 32ull * j) * E;
+        if (off + E <= a.span) consume(a, off, (T)*q, h);
+        q += 32;
+    }
 }
 
 template <class T, bool APTR>
@@ -105,43 +158,24 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
             const bool whole = (u + 1) * a.unit <= a.span;
             if constexpr (APTR) {
                 ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
-                uint32_t j = 0;
-                if (whole) {
-                    for (; j + TILE <= per_unit; j += TILE) {
-                        T v[TILE];
-                        q.read_tile(v, 32);
-#pragma unroll
-                        for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
-                        /* advance after the values are used: a page-leaving
-                         * step then unlinks with no loads still in flight */
-                        q += 32 * TILE;
+                if (a.access == AP_ACCESS_DEREF) {
+                    seq_unit_deref<T>(q, a, e0, per_unit, h);
+                } else if (a.access == AP_ACCESS_RANGE && whole) {
+                    /* translate once for the unit, then stream plain loads
+                     * through the linked translation (valid while q lives) */
+                    const T* p = q.pin_range(32ull * E * (per_unit - 1) + E);
+                    if (p) {
+                        raw_reader<T> rr{p};
+                        seq_unit<T>(rr, a, e0, per_unit, true, h);
+                    } else {
+                        seq_unit<T>(q, a, e0, per_unit, whole, h);
                     }
-                }
-                for (; j < per_unit; ++j) {
-                    const uint64_t off = (e0 + 32ull * j) * E;
-                    if (off + E <= a.span) consume(a, off, (T)*q, h);
-                    q += 32;
+                } else {
+                    seq_unit<T>(q, a, e0, per_unit, whole, h);
                 }
             } else {
-                const T* q = reinterpret_cast<const T*>(a.raw) + e0;
-                uint32_t j = 0;
-                if (whole) {
-                    for (; j + TILE <= per_unit; j += TILE) {
-                        T v[TILE];
-#pragma unroll
-                        for (int k = 0; k < TILE; ++k) {
-                            v[k] = ap::detail::ld_data<T>(q);
-                            q += 32;
-                        }
-#pragma unroll
-                        for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
-                    }
-                }
-                for (; j < per_unit; ++j) {
-                    const uint64_t off = (e0 + 32ull * j) * E;
-                    if (off + E <= a.span) consume(a, off, ap::detail::ld_data<T>(q), h);
-                    q += 32;
-                }
+                raw_reader<T> q{reinterpret_cast<const T*>(a.raw) + e0};
+                seq_unit<T>(q, a, e0, per_unit, whole, h);
             }
         }
     }
@@ -221,6 +255,8 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
     a->unit = cfg->unit_bytes;
     a->page = cfg->page_bytes;
     a->span = cfg->span_bytes ? cfg->span_bytes : rg.bytes;
+    a->access = cfg->access;
+    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_RANGE) return AP_EINVAL;
     switch (cfg->pattern) {
         case AP_SEQ:
             if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;

@@ -255,6 +255,7 @@ extern "C" int ap_mmap(ap_cache_t c, const void* host_buf, uint64_t bytes, ap_re
     d.npages = npages;
     d.pte = rg.pte;
     d.cache = c->d_cache;
+    d.pool = c->pool;
     d.id = id;
     d.live = 1;
     AP_CUDA_TRY(cudaMemcpy(c->regions + id, &d, sizeof d, cudaMemcpyHostToDevice));

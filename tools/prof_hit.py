@@ -49,11 +49,14 @@ def t(fn, n=5):
     return min(ts), float(np.mean(ts))
 
 
-ta = t(lambda: ap.ap_bench_read(cache, r, cfg, out))
 tr = t(lambda: ap.ap_bench_read(cache, r, cfg_raw, out2))
 nb = span * passes
-print(f"unit={unit} passes={passes} apointer {nb/ta[1]/1e9:.1f} GB/s raw {nb/tr[1]/1e9:.1f} GB/s "
-      f"overhead {ta[1]/tr[1]-1:.3f} equal={bool(torch.equal(out, out2))}")
+for acc, name in ((ap.AP_ACCESS_TILE, "tile"), (ap.AP_ACCESS_RANGE, "range"), (ap.AP_ACCESS_DEREF, "deref")):
+    cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=passes, span_bytes=span,
+                       access=acc)
+    ta = t(lambda: ap.ap_bench_read(cache, r, cfg, out))
+    print(f"unit={unit} passes={passes} {name:5s} apointer {nb/ta[1]/1e9:.1f} GB/s raw {nb/tr[1]/1e9:.1f} GB/s "
+          f"overhead {ta[1]/tr[1]-1:.3f} equal={bool(torch.equal(out, out2))}")
 if do_c2:
     cfg2 = ap.bench_cfg(ap.AP_UNIFORM, 4, 148, 512, reads_per_thread=8, seed=1234)
     ap.ap_cache_reset(cache)
