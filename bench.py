@@ -427,7 +427,7 @@ def main():
     p.add_argument("--steps", type=int, default=5)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--workload", default="c2", choices=["c2", "c4", "c5"])
+    p.add_argument("--workload", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--group", type=int, default=1, help="collage candidates per warp")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -448,6 +448,11 @@ def main():
         res = bench_collage.run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler,
                                         host_link_peak)
         drop = ("got", "is_copy", "src")
+    elif args.workload in ("c1", "c3"):
+        import bench_reads
+        res = bench_reads.run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler,
+                                    host_link_peak, aligned_empty)
+        drop = ()
     else:
         res = run_c2(args, torch, dev, rank, world, dist)
         drop = ("file", "got")
@@ -461,6 +466,8 @@ def main():
     if rank == 0:
         if args.workload in ("c4", "c5"):
             line = bench_collage.emit_collage(args, res_all, world, METRIC)
+        elif args.workload in ("c1", "c3"):
+            line = bench_reads.emit_reads(args, res_all, world, METRIC)
         else:
             line = emit_c2(args, res_all, rank, world)
         print(json.dumps(line), flush=True)

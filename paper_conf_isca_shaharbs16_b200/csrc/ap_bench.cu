@@ -121,6 +121,13 @@ __device__ __forceinline__ void seq_unit(R& q, const BenchArgs& a, uint64_t e0, 
             for (int k = 0; k < TILE; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
             q += 32 * TILE; /* after the values are used: no loads in flight at an unlink */
         }
+        for (; j + TILE / 2 <= per_unit; j += TILE / 2) { /* short units (e.g. 4 KiB pages) */
+            T v[TILE / 2];
+            q.read_tile(v, 32);
+#pragma unroll
+            for (int k = 0; k < TILE / 2; ++k) consume(a, (e0 + 32ull * (j + k)) * E, v[k], h);
+            q += 32 * (TILE / 2);
+        }
     }
     for (; j < per_unit; ++j) {
         const uint64_t off = (e0 + 32ull * j) * E;
