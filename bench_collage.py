@@ -94,18 +94,17 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
                           cfg["w"], pd, bd, off, ids)
     t_index = time.time() - t0
     nb = (cfg["W"] // 32) * (cfg["H"] // 32)
-    b0, b1 = rank * nb // world, (rank + 1) * nb // world
+    from paper_conf_isca_shaharbs16_b200 import mgpu
+    b0, b1 = mgpu.block_range(nb, rank, world)
     tgt_host = torch.from_numpy(img).pin_memory()
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0)
-    gather_list = [torch.empty_like(win) for _ in range(world)] if (rank == 0 and world > 1) else None
-
     def step():
         ap.ap_collage_run(cache, region, inp, win, stream)
         if world > 1:
-            dist.gather(win, gather_list, dst=0)
+            mgpu.gather_winners(win, rank, world, dist, nb)  # one NCCL gather (S12)
 
     link = host_link_peak(torch, dev)
     for _ in range(args.warmup):

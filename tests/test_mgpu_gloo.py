@@ -1,0 +1,74 @@
+"""The N>1 collage path on CPU: two gloo ranks each compute their block range
+(with the oracle -- the GPU kernels are covered by the gpu tests) and gather
+the winners with paper_conf_isca_shaharbs16_b200.mgpu; rank 0 must hold
+exactly the single-process answer."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import synth
+from paper_conf_isca_shaharbs16_b200 import mgpu
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _setup():
+    n, stride, w, bb = 1500, 4096, 2500, 8
+    recs = synth.make_records(n, stride, 7)
+    proj, bias = synth.make_lsh_params(3, 5, w, seed=8)
+    img, _, _ = synth.make_target(224, 96, n, ds_seed=7, seed=9, pool=16, copy_permille=100)
+    off, ids = oracle.build_index(recs, stride, n, proj, bias, w, bb, threads=1)
+    return n, stride, w, bb, recs, proj, bias, img, off, ids
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, stride, w, bb, recs, proj, bias, img, off, ids = _setup()
+    nb = (224 // 32) * (96 // 32)
+    b0, b1 = mgpu.block_range(nb, rank, world)
+    mine = oracle.collage(img, proj, bias, w, bb, recs, stride, n, off, ids, b0=b0, nb=b1 - b0,
+                          threads=1)
+    full = mgpu.gather_winners(torch.from_numpy(mine.view(np.int32)), rank, world, dist, nb)
+    if rank == 0:
+        q.put(full.numpy().view(np.uint32).copy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_partitioned_collage_gathers_the_whole_answer(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    n, stride, w, bb, recs, proj, bias, img, off, ids = _setup()
+    want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, off, ids, threads=1)
+    assert np.array_equal(got, want)
+
+
+def test_block_ranges_cover_exactly():
+    for nb in (1, 7, 21, 1024, 65536):
+        for world in (1, 2, 3, 8):
+            rs = [mgpu.block_range(nb, r, world) for r in range(world)]
+            assert rs[0][0] == 0 and rs[-1][1] == nb
+            assert all(rs[i][1] == rs[i + 1][0] for i in range(world - 1))
+            assert max(b - a for a, b in rs) - min(b - a for a, b in rs) <= 1
