@@ -28,7 +28,7 @@ def collage_config(name):
                     workload="C4: 1M 32x32 RGB tiles (4 GiB file of 4 KiB-padded histograms in "
                              "pinned host memory), 1024x1024 target, LSH L=4 K=8 2^14 buckets, "
                              "integer SSD, 256 MiB page cache (cold per step), 1 B200")
-    return dict(name="c5", N=10_000_000, W=8192, H=8192, L=4, K=8, bb=16, w=60000,
+    return dict(name="c5", N=10_000_000, W=8192, H=8192, L=4, K=8, bb=16, w=40000,
                 frames=524288, page=4096, stride=4096,
                 workload="C5: 10M tiles in a 40.96 GB pinned host file, 8192x8192 target, LSH "
                          "L=4 K=8 2^16 buckets, query blocks partitioned over the ranks, 2 GiB "
