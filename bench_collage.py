@@ -100,7 +100,8 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
-                        cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0)
+                        cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0,
+                        schedule=args.schedule)
     def step():
         ap.ap_collage_run(cache, region, inp, win, stream)
         if world > 1:
@@ -123,14 +124,30 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
             stats.append(ap.ap_cache_stats(cache))
     err = ap.ap_last_device_error(cache)
     got = win.cpu().numpy().view(np.uint32).copy()
+    # the other schedule, for comparison (cold cache, same winners)
+    other = 1 - args.schedule
+    inp_o = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
+                          cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
+                          block_count=b1 - b0, schedule=other)
+    win_o = torch.empty_like(win)
+    t_other = []
+    for _ in range(2):
+        ap.ap_cache_reset(cache)
+        t_other.append(timed(torch, lambda: ap.ap_collage_run(cache, region, inp_o, win_o, stream),
+                             stream))
+    other_stats = ap.ap_cache_stats(cache)
+    other_res = dict(schedule=other, s=min(t_other), major=other_stats["major"],
+                     fill_GB=other_stats["fill_bytes"] / 1e9,
+                     equal=bool(torch.equal(win_o, win)))
 
     # raw twin: identical kernel on a fully resident HBM copy (c4 only: 4 GiB)
     raw = None
     if cfg["name"] == "c4":
         dcopy = torch.from_numpy(recs).to(dev)
         inp_raw = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
-                                cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
-                                block_count=b1 - b0, mode=ap.AP_MODE_RAW, raw_base=dcopy)
+                                        cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
+                                block_count=b1 - b0, mode=ap.AP_MODE_RAW, raw_base=dcopy,
+                                schedule=args.schedule)
         win_raw = torch.empty_like(win)
         for _ in range(2):
             timed(torch, lambda: ap.ap_collage_run(cache, region, inp_raw, win_raw, stream), stream)
@@ -159,6 +176,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         e2e.append(s.elapsed_time(e) * 1e-3)
     cands = None
     res = dict(cfg=cfg, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
+               other=other_res,
                link=link, raw=raw, e2e=e2e, clocks=clk.summary(), t_gen=t_gen, t_pin=t_pin,
                t_index=t_index, h2d=int(tgt_host.numel()), d2h=int(win.numel() * 4),
                is_copy=is_copy, src=src, cands=cands)
@@ -214,6 +232,7 @@ def emit_collage(args, res_all, world, METRIC):
                    "blocks": r0["nb"], "L": cfg["L"], "K": cfg["K"], "bucket_bits": cfg["bb"],
                    "w": cfg["w"], "cache_bytes_per_gpu": cfg["frames"] * cfg["page"],
                    "group": args.group,
+                   "schedule": "lsh-sorted blocks" if args.schedule else "natural order",
                    "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",
                    "parallelism": f"blocks partitioned over {world} rank(s) + NCCL gather"},
         "collage": {"blocks_rank0": r0["b1"] - r0["b0"], "major_faults": st["major"],
@@ -222,7 +241,9 @@ def emit_collage(args, res_all, world, METRIC):
                     "device_error": r0["err"], "setup_s": {"generate": round(r0["t_gen"], 2),
                                                           "pin": round(r0["t_pin"], 2),
                                                           "index_build_gpu": round(r0["t_index"], 3)},
-                    "per_rank_s": [round(sum(r["times"]) / args.steps, 6) for r in res_all]},
+                    "per_rank_s": [round(sum(r["times"]) / args.steps, 6) for r in res_all],
+                    "other_schedule": {k: (round(v, 6) if isinstance(v, float) else v)
+                                       for k, v in r0["other"].items()}},
         "roofline": {"bound": "host_link", "achieved": round(fill / t0 / 1e9, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
                      "frac": round(fill / t0 / 1e9 / r0["link"], 4),

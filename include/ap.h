@@ -206,7 +206,16 @@ typedef struct {
     uint64_t block_count;        /* number of query blocks                        */
     int32_t mode;                /* AP_MODE_APOINTER | AP_MODE_RAW                 */
     const void* raw_base;        /* AP_MODE_RAW: device-readable record file       */
+    int32_t schedule;            /* AP_SCHED_NATURAL: CTA i = block i (the paper's *
+                                  * single kernel); AP_SCHED_LSH: blocks are first *
+                                  * sorted by their LSH keys (an extra key kernel  *
+                                  * + radix sort) so blocks sharing buckets run    *
+                                  * together and reuse cached records.  Results   *
+                                  * are identical (per-block argmin).             */
 } ap_collage_in;
+
+#define AP_SCHED_NATURAL 0
+#define AP_SCHED_LSH 1
 
 /* ap_collage_run — the collage kernel ("calculates the
  * histogram of each 32x32 block, computes its LSH keys, reads the candidate

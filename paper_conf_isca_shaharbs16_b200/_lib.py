@@ -16,6 +16,7 @@ AP_POLICY_CLOCK, AP_POLICY_RANDOM = 0, 1
 AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
 AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE = 0, 1, 2
+AP_SCHED_NATURAL, AP_SCHED_LSH = 0, 1
 
 u64, u32, i32, vp, ci = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int
 
@@ -40,7 +41,7 @@ class ap_collage_in(ctypes.Structure):
                 ("bucket_bits", u32), ("w", i32), ("proj_dev", vp), ("bias_dev", vp),
                 ("offsets_dev", vp), ("ids_dev", vp), ("N", u64), ("rec_stride", u32),
                 ("group", u32), ("block_begin", u64), ("block_count", u64), ("mode", i32),
-                ("raw_base", vp)]
+                ("raw_base", vp), ("schedule", i32)]
 
 
 class APError(RuntimeError):

@@ -40,6 +40,8 @@ struct ap_cache_s {
     ap::dev_cache h{};                /* host mirror         */
     std::vector<ap_region_host> reg;
     int num_sms = 148;
+    void* scratch = nullptr; /* grown on demand (collage schedule) */
+    size_t scratch_bytes = 0;
 };
 
 /* Switch to the cache's device for the lifetime of the guard. */
@@ -66,6 +68,8 @@ struct ap_device_guard {
     } while (0)
 
 void ap_note_cuda_error(cudaError_t e, const char* what, const char* file, int line);
+/* Scratch device memory of at least `bytes` (synchronises only when it grows). */
+void* ap_scratch(ap_cache_s* c, size_t bytes);
 bool ap_region_ok(const ap_cache_s* c, ap_region_t r);
 
 #endif

@@ -37,6 +37,20 @@ extern "C" const char* ap_version(void) {
     return "apointer-b200 0.1 (sm_100a; long apointer, no TLB, clock eviction)";
 }
 
+void* ap_scratch(ap_cache_s* c, size_t bytes) {
+    if (c->scratch_bytes >= bytes) return c->scratch;
+    cudaDeviceSynchronize();
+    cudaFree(c->scratch);
+    c->scratch = nullptr;
+    c->scratch_bytes = 0;
+    if (cudaMalloc(&c->scratch, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    c->scratch_bytes = bytes;
+    return c->scratch;
+}
+
 bool ap_region_ok(const ap_cache_s* c, ap_region_t r) {
     return c && r < c->reg.size() && c->reg[r].live;
 }
@@ -195,6 +209,7 @@ extern "C" int ap_cache_destroy(ap_cache_t c) {
     cudaFree(c->regions);
     cudaFree(c->stats);
     cudaFree(c->d_cache);
+    cudaFree(c->scratch);
     delete c;
     return AP_OK;
 }

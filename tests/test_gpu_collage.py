@@ -48,9 +48,9 @@ def test_index_matches_oracle(ap, K, bb):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group", [1, 2, 4])
+@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1)])
 @pytest.mark.parametrize("frames", [48, 5000])
-def test_collage_matches_oracle(ap, group, frames):
+def test_collage_matches_oracle(ap, group, schedule, frames):
     dev = torch.device("cuda:0")
     n, stride, w, bb, L, K = 4096, 4096, 2500, 9, 4, 6
     W, H = 512, 256
@@ -62,7 +62,8 @@ def test_collage_matches_oracle(ap, group, frames):
         tgt = torch.from_numpy(img).to(dev)
         nb = (W // 32) * (H // 32)
         win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
-        inp = ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride, group=group)
+        inp = ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride, group=group,
+                            schedule=schedule)
         ap.ap_collage_run(cache, r, inp, win)
         torch.cuda.synchronize()
         assert ap.ap_last_device_error(cache) == 0
@@ -77,7 +78,7 @@ def test_collage_matches_oracle(ap, group, frames):
         rawd = torch.from_numpy(recs).to(dev)
         win2 = torch.zeros_like(win)
         inp2 = ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride, group=group,
-                             mode=ap.AP_MODE_RAW, raw_base=rawd)
+                             mode=ap.AP_MODE_RAW, raw_base=rawd, schedule=schedule)
         ap.ap_collage_run(cache, r, inp2, win2)
         torch.cuda.synchronize()
         assert np.array_equal(win2.cpu().numpy().view(np.uint32), want)
@@ -106,7 +107,8 @@ def test_collage_partitioned_blocks_equal_whole(ap):
             b0, b1 = g * nb // 3, (g + 1) * nb // 3
             part = torch.zeros((b1 - b0, 2), dtype=torch.int32, device=dev)
             ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
-                                                      block_begin=b0, block_count=b1 - b0), part)
+                                                      block_begin=b0, block_count=b1 - b0,
+                                                      schedule=g % 2), part)
             parts.append(part)
         assert torch.equal(torch.cat(parts), full)
         ap.ap_munmap(cache, r)
