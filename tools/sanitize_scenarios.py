@@ -1,0 +1,88 @@
+"""Small scenarios for compute-sanitizer (memcheck / racecheck / synccheck):
+every fault-path branch (minor, major, eviction, exhaustion back-off,
+divergent groups, partial warps, tiles straddling pages) on tiny inputs,
+each checked against the oracle so a sanitizer run is also a parity run."""
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, ".")
+sys.path.insert(0, "tests")
+import oracle  # noqa: E402
+import paper_conf_isca_shaharbs16_b200 as ap  # noqa: E402
+import synth  # noqa: E402
+from helpers import check_invariants, make_file, make_records  # noqa: E402
+
+dev = torch.device("cuda:0")
+ok = True
+
+
+def check(name, cond):
+    global ok
+    print(f"{name}: {'ok' if cond else 'FAIL'}", flush=True)
+    ok &= bool(cond)
+
+
+f = make_file((1 << 20) + 4096 * 3 + 48, 1)
+for frames, policy in ((2, 0), (8, 1)):
+    c = ap.ap_cache_create(frames, 4096)
+    ap.ap_cache_set_policy(c, policy, 3)
+    r = ap.ap_mmap(c, f)
+    n = f.nbytes
+    out = torch.zeros(n, dtype=torch.uint8, device=dev)
+    ap.ap_bench_read(c, r, ap.bench_cfg(ap.AP_SEQ, 16, 2, 64, unit_bytes=4096, out_copy=True,
+                                        span_bytes=n), out)
+    torch.cuda.synchronize()
+    whole = n // 16 * 16
+    check(f"seq copy frames={frames}", np.array_equal(out.cpu().numpy()[:whole], f[:whole]))
+    ck = torch.zeros(256, dtype=torch.int64, device=dev)
+    ap.ap_bench_read(c, r, ap.bench_cfg(ap.AP_UNIFORM, 4, 2, 128, reads_per_thread=3, seed=5), ck)
+    torch.cuda.synchronize()
+    check(f"uniform frames={frames}", np.array_equal(ck.cpu().numpy().view(np.uint64),
+                                                     oracle.read_uniform(f, n, 4, 256, 3, 5)))
+    nd = 64 * 4096
+    ap.ap_bench_read(c, r, ap.bench_cfg(ap.AP_DIVERGENT, 16, 2, 128, reads_per_thread=2,
+                                        page_bytes=4096, seed=9), ck)
+    torch.cuda.synchronize()
+    check(f"divergent frames={frames}", np.array_equal(
+        ck.cpu().numpy().view(np.uint64), oracle.read_divergent(f, n, 4096, 16, 256, 2, 9)))
+    for acc in (ap.AP_ACCESS_DEREF, ap.AP_ACCESS_RANGE):
+        ck2 = torch.zeros(128, dtype=torch.int64, device=dev)
+        ap.ap_bench_read(c, r, ap.bench_cfg(ap.AP_SEQ, 16, 1, 128, unit_bytes=4096, access=acc), ck2)
+        torch.cuda.synchronize()
+        check(f"seq access={acc} frames={frames}", np.array_equal(
+            ck2.cpu().numpy().view(np.uint64), oracle.read_seq(f, n, 4096, 16, 128, 1)))
+    check(f"invariants frames={frames}", check_invariants(ap, c, [r], frames) == [])
+    check(f"device error frames={frames}", ap.ap_last_device_error(c) == 0)
+    ap.ap_munmap(c, r)
+    ap.ap_cache_destroy(c)
+
+# collage: groups 1/2/4 over a 12-frame cache, both schedules, unaligned-free
+n, stride, w, bb = 512, 4096, 2500, 6
+recs = make_records(n, stride, 3)
+proj, bias = synth.make_lsh_params(2, 4, w, seed=4)
+img, _, _ = synth.make_target(128, 64, n, ds_seed=3, seed=5, pool=4, copy_permille=100)
+c = ap.ap_cache_create(12, 4096)
+r = ap.ap_mmap(c, recs)
+off = torch.zeros((2, (1 << bb) + 1), dtype=torch.int32, device=dev)
+ids = torch.zeros((2, n), dtype=torch.int32, device=dev)
+pd, bd = torch.from_numpy(proj).to(dev), torch.from_numpy(bias).to(dev)
+ap.ap_lsh_build_index(c, r, n, stride, 2, 4, bb, w, pd, bd, off, ids)
+o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+check("index", np.array_equal(off.cpu().numpy().view(np.uint32), o_off))
+want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+tgt = torch.from_numpy(img).to(dev)
+for g in (1, 2, 4):
+    for sch in (0, 1):
+        win = torch.zeros((8, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(c, r, ap.collage_in(tgt, 128, 64, pd, bd, w, bb, off, ids, n, group=g,
+                                              schedule=sch), win)
+        torch.cuda.synchronize()
+        check(f"collage group={g} schedule={sch}",
+              np.array_equal(win.cpu().numpy().view(np.uint32), want))
+check("collage invariants", check_invariants(ap, c, [r], 12) == [])
+ap.ap_munmap(c, r)
+ap.ap_cache_destroy(c)
+print("ALL OK" if ok else "FAILURES")
+sys.exit(0 if ok else 1)
