@@ -572,16 +572,70 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
 template <class T, int N>
 struct tile_out {
     T v[N];
+    uint64_t x; /* the pointer's translation afterwards (unlinked) */
 };
 
-/* Element-wise tile read for tiles that straddle a page: each element goes
- * through a temporary unlinked pointer (fault, read, unlink). */
+/* Tile read for tiles that straddle a page boundary (e.g. unaligned 3 KiB
+ * records).  Lanes are linked on entry.  A tile spanning at
+ * most two pages: the elements in the linked page are loaded, the link is
+ * dropped (so the lane holds no pin while faulting, R-A19), the lanes whose
+ * tile continues link the next page through a temporary pointer, load the
+ * rest, and unlink it.  Longer tiles go element by element.  The pointer
+ * ends unlinked (it still designates the same offset). */
 template <class T, int N>
 __device__ AP_SLOW_ATTR tile_out<T, N> read_tile_slow(unsigned m, uint64_t x, uint64_t page,
                                                       const dev_region* r, uint32_t lg,
                                                       int64_t stride) {
     tile_out<T, N> t;
-    const uint64_t f0 = (x >> 63) ? ((page << lg) | (x & ((1ull << lg) - 1))) : x;
+    const uint64_t P = 1ull << lg;
+    const uint64_t f0 = (x >> 63) ? ((page << lg) | (x & (P - 1))) : x;
+    const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
+    const bool two = stride > 0 && span < P && (x >> 63);
+    if (__all_sync(m, two)) {
+        const uint64_t next = ((f0 >> lg) + 1) << lg;
+        const T* a = reinterpret_cast<const T*>(x & XL_ADDR);
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
+            const uint64_t fk = f0 + (uint64_t)(k * stride * (int64_t)sizeof(T));
+            t.v[k] = fk < next ? ld_data<T>(a + k * stride) : T{};
+        }
+        unlink_lanes(m, true, r, page); /* release: orders the loads above first */
+        const bool cross = f0 + span + sizeof(T) > next;
+        if (cross) {
+            const unsigned mc = __activemask();
+            const slow_out<T> o = deref_slow<T>(mc, next, 0, r);
+            const bool l = (o.x >> 63) != 0;
+            if (l) {
+                const T* b = reinterpret_cast<const T*>(o.x & XL_ADDR);
+#pragma unroll
+                for (int k = 0; k < N; ++k) {
+                    const uint64_t fk = f0 + (uint64_t)(k * stride * (int64_t)sizeof(T));
+                    if (fk >= next) t.v[k] = ld_data<T>(b + (fk - next) / sizeof(T));
+                }
+            }
+            if (__any_sync(mc, l)) unlink_lanes(mc, l, r, o.page);
+            if (!l) {
+                /* the fault path dropped this lane's link under frame
+                 * pressure (its value is in o.val): element by element */
+#pragma unroll 1
+                for (int k = 0; k < N; ++k) {
+                    const uint64_t fk = f0 + (uint64_t)(k * stride * (int64_t)sizeof(T));
+                    if (fk >= next) {
+                        const unsigned mk = __activemask();
+                        const slow_out<T> e = deref_slow<T>(mk, fk, 0, r);
+                        t.v[k] = e.val;
+                        const bool le = (e.x >> 63) != 0;
+                        if (__any_sync(mk, le)) unlink_lanes(mk, le, r, e.page);
+                    }
+                }
+            }
+        }
+        __syncwarp(m); /* reconverge the lanes that went through phase 2 */
+        t.x = f0;
+        return t;
+    }
+    /* general case: each element through a temporary pointer */
+    if (__any_sync(m, (x >> 63) != 0)) unlink_lanes(m, (x >> 63) != 0, r, page);
     for (int k = 0; k < N; ++k) {
         const uint64_t fk = f0 + (uint64_t)(k * stride * (int64_t)sizeof(T));
         const slow_out<T> o = deref_slow<T>(m, fk, 0, r);
@@ -589,6 +643,7 @@ __device__ AP_SLOW_ATTR tile_out<T, N> read_tile_slow(unsigned m, uint64_t x, ui
         const bool l = (o.x >> 63) != 0;
         if (__any_sync(m, l)) unlink_lanes(m, l, r, o.page);
     }
+    t.x = f0;
     return t;
 }
 
@@ -693,11 +748,11 @@ struct ptr {
             }
             ok = linked() && ((x ^ (x + span)) >> lg) == 0;
             if (!__all_sync(m, ok)) {
-                /* hold no pin while the element-wise path faults (R-A19) */
-                release();
+                /* some lane's tile straddles a page */
                 const detail::tile_out<T, N> t = detail::read_tile_slow<T, N>(m, x, page, r, lg, stride);
 #pragma unroll
                 for (int k = 0; k < N; ++k) v[k] = t.v[k];
+                x = t.x;
                 return;
             }
         }

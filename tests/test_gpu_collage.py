@@ -13,7 +13,7 @@ from helpers import check_invariants, make_records
 pytestmark = pytest.mark.gpu
 
 
-def _setup(n, W, H, L, K, w, bb, seed=21, stride=4096, frames=256, page=4096):
+def _setup(n, W, H, L, K, w, bb, seed=21, stride=4096, frames=256, page=4096):  # noqa: ARG001
     recs = make_records(n, stride, seed)
     proj, bias = synth.make_lsh_params(L, K, w, seed=seed + 1)
     img, src, is_copy = synth.make_target(W, H, n, ds_seed=seed, seed=seed + 2, pool=32,
@@ -111,6 +111,38 @@ def test_collage_partitioned_blocks_equal_whole(ap):
                                                       schedule=g % 2), part)
             parts.append(part)
         assert torch.equal(torch.cat(parts), full)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("group", [1, 2, 4])
+@pytest.mark.parametrize("frames", [40, 3000])
+def test_unaligned_records_collage(ap, group, frames):
+    """NEXT N1: 3 KiB histograms without padding, so records
+    straddle 4 KiB pages; the same kernel and pointers must still match the
+    oracle bit for bit."""
+    dev = torch.device("cuda:0")
+    n, stride, w, bb, L, K = 4096, 3072, 2500, 9, 4, 6
+    W, H = 384, 256
+    recs, proj, bias, img, src, is_copy = _setup(n, W, H, L, K, w, bb, stride=stride)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        assert np.array_equal(off.cpu().numpy().view(np.uint32), o_off)
+        assert np.array_equal(ids.cpu().numpy().view(np.uint32), o_ids)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride,
+                                                  group=group), win)
+        torch.cuda.synchronize()
+        assert ap.ap_last_device_error(cache) == 0
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+        assert np.array_equal(win.cpu().numpy().view(np.uint32), want)
+        assert check_invariants(ap, cache, [r], frames) == []
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)

@@ -84,5 +84,21 @@ for g in (1, 2, 4):
 check("collage invariants", check_invariants(ap, c, [r], 12) == [])
 ap.ap_munmap(c, r)
 ap.ap_cache_destroy(c)
+# unaligned 3 KiB records (tiles straddle pages)
+recs3 = make_records(n, 3072, 3)
+c = ap.ap_cache_create(6, 4096)
+r = ap.ap_mmap(c, recs3)
+ap.ap_lsh_build_index(c, r, n, 3072, 2, 4, bb, w, pd, bd, off, ids)
+o_off, o_ids = oracle.build_index(recs3, 3072, n, proj, bias, w, bb)
+want = oracle.collage(img, proj, bias, w, bb, recs3, 3072, n, o_off, o_ids)
+for g in (1, 4):
+    win = torch.zeros((8, 2), dtype=torch.int32, device=dev)
+    ap.ap_collage_run(c, r, ap.collage_in(tgt, 128, 64, pd, bd, w, bb, off, ids, n, 3072, group=g),
+                      win)
+    torch.cuda.synchronize()
+    check(f"unaligned collage group={g}", np.array_equal(win.cpu().numpy().view(np.uint32), want))
+check("unaligned invariants", check_invariants(ap, c, [r], 6) == [])
+ap.ap_munmap(c, r)
+ap.ap_cache_destroy(c)
 print("ALL OK" if ok else "FAILURES")
 sys.exit(0 if ok else 1)
