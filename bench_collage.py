@@ -21,7 +21,15 @@ GiB = 1 << 30
 LSH_SEED, DS_SEED, TGT_SEED = 22, 21, 23
 
 
-def collage_config(name):
+def collage_config(name, stride=4096):
+    cfg = _collage_config(name)
+    if stride != 4096:  # NEXT N1: unaligned 3 KiB records, no padding
+        cfg["stride"] = stride
+        cfg["workload"] += f"; UNALIGNED {stride}-B records (no padding, records straddle pages)"
+    return cfg
+
+
+def _collage_config(name):
     if name == "c4":
         return dict(name="c4", N=1 << 20, W=1024, H=1024, L=4, K=8, bb=14, w=60000,
                     frames=65536, page=4096, stride=4096,
@@ -67,7 +75,7 @@ def _shm_records(cfg, rank, world, dist):
 def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_link_peak):
     import paper_conf_isca_shaharbs16_b200 as ap
     import synth
-    cfg = collage_config(args.workload)
+    cfg = collage_config(args.workload, args.stride)
     stream = torch.cuda.current_stream()
     t0 = time.time()
     if cfg["name"] == "c4":
@@ -231,6 +239,7 @@ def emit_collage(args, res_all, world, METRIC):
         "config": {"workload": cfg["workload"], "records": cfg["N"], "target": [cfg["W"], cfg["H"]],
                    "blocks": r0["nb"], "L": cfg["L"], "K": cfg["K"], "bucket_bits": cfg["bb"],
                    "w": cfg["w"], "cache_bytes_per_gpu": cfg["frames"] * cfg["page"],
+                   "record_stride": cfg["stride"],
                    "group": args.group,
                    "schedule": "lsh-sorted blocks" if args.schedule else "natural order",
                    "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",

@@ -188,6 +188,15 @@ int ap_bench_read(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg,
 int ap_bench_read_host(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg,
                        void* out_host, double* seconds);
 
+/* ap_bench_latency — Table I analogue: one warp, all
+ * lanes on one (prefilled) page, coalesced 4-B accesses; op = 0 raw read,
+ * 1 apointer read, 2 raw increment, 3 apointer increment, 4 raw read+inc,
+ * 5 apointer read+inc.  cycles[0] = mean clock64 cycles per op after
+ * subtracting cycles[1], the cost of an empty timing pair.  The raw pointer
+ * reads the same frame the apointer is linked to.  Synchronises. */
+int ap_bench_latency(ap_cache_t cache, ap_region_t region, int op, uint32_t reps,
+                     uint64_t* cycles);
+
 /* ---------------------------------------------------- photo collage (§VI-E) */
 typedef struct {
     const uint8_t* target_dev;   /* W*H*3 uint8 RGB, interleaved, row-major       */

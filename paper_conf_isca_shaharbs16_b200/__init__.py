@@ -158,6 +158,13 @@ def ap_bench_read_host(cache, region, cfg, out_host):
     return sec.value
 
 
+def ap_bench_latency(cache, region, op, reps=1000):
+    """Returns (cycles per op, empty timing-pair cycles)."""
+    out = (ctypes.c_uint64 * 2)()
+    _lib.check("ap_bench_latency", _lib.lib().ap_bench_latency(cache, region, op, reps, out))
+    return int(out[0]), int(out[1])
+
+
 def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev, ids_dev, N,
                rec_stride=4096, group=1, block_begin=0, block_count=None,
                mode=AP_MODE_APOINTER, raw_base=None, L=None, K=None, schedule=1):

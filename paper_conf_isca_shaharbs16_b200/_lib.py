@@ -82,6 +82,7 @@ def lib():
             "ap_bench_read_host": (ci, [vp, u32, ctypes.POINTER(ap_bench_cfg), vp,
                                         ctypes.POINTER(ctypes.c_double)]),
             "ap_collage_run": (ci, [vp, u32, ctypes.POINTER(ap_collage_in), vp, vp]),
+            "ap_bench_latency": (ci, [vp, u32, ci, u32, ctypes.POINTER(u64)]),
             "ap_lsh_build_index": (ci, [vp, u32, u64, u32, u32, u32, u32, i32, vp, vp, vp, vp,
                                         vp]),
         }
@@ -97,7 +98,8 @@ EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", 
             "ap_munmap", "ap_region_devptr", "ap_region_npages", "ap_cache_stats",
             "ap_cache_reset", "ap_cache_set_policy", "ap_cache_set_tuning",
             "ap_last_device_error", "ap_cache_dump", "ap_region_dump_pte", "ap_prefill",
-            "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index"]
+            "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index",
+            "ap_bench_latency"]
 
 
 def check(fn, rc):

@@ -329,3 +329,122 @@ extern "C" int ap_bench_read_host(ap_cache_t c, ap_region_t region, const ap_ben
     cudaFree(d);
     return rc;
 }
+
+/* ------------------------------------------------------------------------
+ * Latency microbenchmark (NEXT N4; the paper's Table I):
+ * one warp, all lanes on one page, coalesced 4-B accesses; cycles per
+ * operation from clock64() around each op, minus the cost of an empty
+ * timing pair (the paper subtracts 16 cycles of measurement overhead). */
+namespace {
+
+__device__ __forceinline__ uint64_t clk() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t)::"memory");
+    return t;
+}
+/* fold v into a live accumulator with a real instruction: the clock read
+ * after it cannot issue before v has arrived */
+#define SINK(v) asm volatile("add.u32 %0, %0, %1;" : "+r"(acc) : "r"((uint32_t)(v)) : "memory")
+/* raw ops as volatile PTX so the compiler cannot hoist or fold them */
+__device__ __forceinline__ uint32_t raw_ld(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void raw_add(const uint32_t*& p, int64_t d) {
+    uint64_t a = (uint64_t)p;
+    asm volatile("add.s64 %0, %0, %1;" : "+l"(a) : "l"(d * 4));
+    p = (const uint32_t*)a;
+}
+
+__global__ void k_latency(const ap::dev_cache* __restrict__ c, uint32_t region, const uint32_t* raw,
+                          int op, uint32_t reps, unsigned long long* out) {
+    /* Each op is repeated `reps` times as a dependent chain between two
+     * clock reads: the next read's address depends on the value just read
+     * (an index inside the same page), so the reads cannot overlap and the
+     * per-op time is the latency (pointer chasing).  Increments chain through
+     * the pointer itself. */
+    const unsigned lane = threadIdx.x & 31;
+    ap::ptr<uint32_t> q = ap::gvmmap<uint32_t>(c, region, 4 * lane);
+    const uint32_t* p = raw + lane;
+    uint32_t acc = *q; /* links q (the page was prefilled: a minor fault) */
+    acc += __ldcg(p);
+    uint32_t v = acc;
+    const uint64_t e0 = clk();
+    SINK(v);
+    const uint64_t e1 = clk();
+    uint64_t t0 = 0, t1 = 0;
+    switch (op) {
+        case 0: /* raw read */
+            t0 = clk();
+            for (uint32_t i = 0; i < reps; ++i) v = raw_ld(p + 32 * (v & 7));
+            SINK(v);
+            t1 = clk();
+            break;
+        case 1: /* apointer read through the register translation */
+            t0 = clk();
+            for (uint32_t i = 0; i < reps; ++i) v = q[(int64_t)(32 * (v & 7))];
+            SINK(v);
+            t1 = clk();
+            break;
+        case 2: /* raw increment (stays in the page) */
+            t0 = clk();
+            for (uint32_t i = 0; i < reps; ++i) raw_add(p, (i & 1) ? -32 : 32);
+            SINK((uint32_t)(uintptr_t)p);
+            t1 = clk();
+            break;
+        case 3: /* apointer increment (stays in the page) */
+            t0 = clk();
+            for (uint32_t i = 0; i < reps; ++i) q += (i & 1) ? -32 : 32;
+            SINK((uint32_t)q.x);
+            t1 = clk();
+            break;
+        case 4: /* raw read + increment */
+            t0 = clk();
+            for (uint32_t i = 0; i < reps; ++i) {
+                v = raw_ld(p + 32 * (v & 1));
+                raw_add(p, (i & 1) ? -32 : 32);
+            }
+            SINK(v);
+            t1 = clk();
+            break;
+        default: /* apointer read + increment */
+            t0 = clk();
+            for (uint32_t i = 0; i < reps; ++i) {
+                v = q[(int64_t)(32 * (v & 1))];
+                q += (i & 1) ? -32 : 32;
+            }
+            SINK(v);
+            t1 = clk();
+            break;
+    }
+    acc += v;
+    if (lane == 0) {
+        const uint64_t empty = e1 - e0;
+        out[0] = (t1 - t0 - empty) / (reps ? reps : 1);
+        out[1] = empty;
+        out[2] = acc;
+    }
+}
+
+}  // namespace
+
+extern "C" int ap_bench_latency(ap_cache_t c, ap_region_t region, int op, uint32_t reps,
+                                uint64_t* cycles) {
+    if (!ap_region_ok(c, region) || op < 0 || op > 5 || !cycles) return AP_EINVAL;
+    if (c->reg[region].bytes < c->page + 256) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    int rc = ap_prefill(c, region, 0, 1, nullptr);
+    if (rc) return rc;
+    unsigned long long* d = nullptr;
+    AP_CUDA_TRY(cudaMalloc(&d, 3 * sizeof(unsigned long long)));
+    k_latency<<<1, 32>>>(c->d_cache, region, (const uint32_t*)c->pool, op, reps, d);
+    cudaError_t e = cudaGetLastError();
+    unsigned long long h[3] = {0, 0, 0};
+    if (e == cudaSuccess) e = cudaMemcpy(h, d, sizeof h, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    AP_CUDA_TRY(e);
+    cycles[0] = h[0];
+    cycles[1] = h[1];
+    return AP_OK;
+}
