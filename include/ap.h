@@ -42,6 +42,7 @@ extern "C" {
 #define AP_EFAULT (-6)    /* device: dereference past the region or misaligned */
 #define AP_ENOFRAME (-7)  /* device: no evictable frame (all pinned)         */
 #define AP_ETIMEDOUT (-8) /* device: fault-path watchdog expired             */
+#define AP_EPERM (-9)     /* device: store through a read-only mapping       */
 
 /* Human-readable text for an AP_* code (static storage, never NULL). */
 const char* ap_strerror(int code);
@@ -52,7 +53,7 @@ typedef uint32_t ap_region_t;
 
 /* ap_cache_create — the GPU page cache (§V "page cache in
  * GPU memory"; frames of page_size bytes, PAPER.md:363 uses 4 KB).
- *   frames     number of page frames, 1 <= frames < 2^29
+ *   frames     number of page frames, 1 <= frames < 2^28
  *   page_size  bytes per page: a power of two in [4096, 2 MiB]
  *   device     CUDA device ordinal
  * Allocates frames*page_size bytes of HBM (page_size aligned), the frame
@@ -75,6 +76,23 @@ int ap_cache_destroy(ap_cache_t cache);
  * Errors: AP_EINVAL (NULL, 0 bytes, misaligned), AP_ERANGE (65535 regions
  * mapped, or > 2^48 pages), AP_ENOMEM, AP_ECUDA. */
 int ap_mmap(ap_cache_t cache, const void* host_buf, uint64_t bytes, ap_region_t* out);
+
+/* ap_mmap_prot — as ap_mmap with protection bits (NEXT N3; PAPER.md:134
+ * Fig. 3 writes `*ptr = 25` through an apointer; "rw").
+ *   prot  AP_PROT_READ, optionally | AP_PROT_WRITE.  A writable mapping
+ *         registers the host bytes without the read-only flag; stores mark
+ *         pages DIRTY and dirty pages are written back to host_buf when they
+ *         are evicted, by ap_msync, ap_munmap and ap_cache_reset.
+ * Errors: as ap_mmap; AP_EINVAL for other prot bits. */
+#define AP_PROT_READ 1
+#define AP_PROT_WRITE 2
+int ap_mmap_prot(ap_cache_t cache, const void* host_buf, uint64_t bytes, int prot,
+                 ap_region_t* out);
+
+/* ap_msync — write every dirty resident page of a writable region back to
+ * its host bytes and mark it clean (synchronises; no kernel may be using the
+ * region).  No-op for read-only regions. */
+int ap_msync(ap_cache_t cache, ap_region_t region);
 
 /* Unmap: frames holding the region's pages go back to the free list.
  * AP_EBUSY if any page of the region still has a positive reference count
@@ -128,7 +146,8 @@ int ap_last_device_error(ap_cache_t cache);
  *   owner_host[frames]  0 = none, else ((region+1) << 48) | page
  *   free_left           frames still on the free list
  *   pte_host[npages]    bits 63:62 state (0 EMPTY, 1 LOADING, 2 VALID),
- *                       61 reference bit, 60:32 frame, 31:0 reference count */
+ *                       61 reference bit, 60 dirty, 59:32 frame,
+ *                       31:0 reference count */
 int ap_cache_dump(ap_cache_t cache, uint64_t* owner_host, uint64_t* free_left);
 int ap_region_npages(ap_cache_t cache, ap_region_t region, uint64_t* npages);
 int ap_region_dump_pte(ap_cache_t cache, ap_region_t region, uint64_t* pte_host);
@@ -187,6 +206,22 @@ int ap_bench_read(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg,
  * launch + device->host copy measured with CUDA events. */
 int ap_bench_read_host(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg,
                        void* out_host, double* seconds);
+
+/* ap_bench_write — stores through apointers into a writable region (NEXT
+ * N3, Fig. 3 `*ptr = 25`).  cfg: pattern AP_SEQ (every element of
+ * [0, span) once, warp units as ap_bench_read) or AP_UNIFORM (race-free
+ * permutation: element (t*R+i)*a mod M, a = the odd number nearest below
+ * 0.618*M coprime with M; needs grid*block*R <= M <= 2^32);
+ * value at element e = low bytes of sm64(seed ^ e) (16-B: sm64(seed^2e),
+ * sm64(seed^(2e+1))).  The host bytes change once the pages are written back
+ * (eviction, ap_msync, ap_munmap).  Asynchronous on `stream`. */
+int ap_bench_write(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg, void* stream);
+
+/* ap_bench_copy — dst[e] = src[e] for the SEQ pattern of cfg, reading and
+ * writing through apointers (the copy kernel of PAPER.md:310-316).  dst must
+ * be writable.  Asynchronous on `stream`. */
+int ap_bench_copy(ap_cache_t cache, ap_region_t src, ap_region_t dst, const ap_bench_cfg* cfg,
+                  void* stream);
 
 /* ap_bench_latency — Table I analogue: one warp, all
  * lanes on one (prefilled) page, coalesced 4-B accesses; op = 0 raw read,

@@ -48,6 +48,9 @@
 
 #include <cuda_runtime.h>
 #include <stdint.h>
+#ifdef AP_DEBUG
+#include <cstdio>
+#endif
 
 /* The fault path is kept out of line by default so the hit path stays a
  * handful of instructions; -DAP_SLOW_INLINE inlines it. */
@@ -62,18 +65,23 @@
 namespace ap {
 
 /* ------------------------------------------------------------ layouts */
-/* Page-table entry (R-A17): [63:62] state, [61] reference bit,
- * [60:32] frame, [31:0] reference count. */
+/* Page-table entry (R-A17): [63:62] state, [61] reference bit, [60] dirty,
+ * [59:32] frame, [31:0] reference count. */
 constexpr uint64_t PTE_EMPTY = 0ull;
 constexpr uint64_t PTE_LOADING = 1ull << 62;
 constexpr uint64_t PTE_VALID = 2ull << 62;
 constexpr uint64_t PTE_REF = 1ull << 61;
-constexpr uint64_t PTE_FRAME_MASK = (1ull << 29) - 1;
+constexpr uint64_t PTE_DIRTY = 1ull << 60; /* writable mappings: frame differs from the file */
+constexpr uint64_t PTE_FRAME_MASK = (1ull << 28) - 1;
 constexpr uint64_t PTE_RC_MASK = 0xffffffffull;
 
 /* Translation field (R-A16). */
 constexpr uint64_t XL_VALID = 1ull << 63;
+constexpr uint64_t XL_DIRTY = 1ull << 62; /* permission-bit slot: this link already set DIRTY */
 constexpr uint64_t XL_ADDR = (1ull << 61) - 1;
+
+constexpr uint32_t PROT_READ = 1;
+constexpr uint32_t PROT_WRITE = 2;
 
 constexpr uint64_t PAGE_MASK48 = (1ull << 48) - 1;
 
@@ -81,6 +89,7 @@ constexpr uint64_t PAGE_MASK48 = (1ull << 48) - 1;
 constexpr int ERR_FAULT = -6;
 constexpr int ERR_NOFRAME = -7;
 constexpr int ERR_TIMEDOUT = -8;
+constexpr int ERR_PERM = -9;
 
 constexpr int POLICY_CLOCK = 0;
 constexpr int POLICY_RANDOM = 1;
@@ -103,7 +112,8 @@ struct alignas(64) dev_region {
     uint32_t id;            /* region id (< 65535)                        */
     uint32_t live;          /* 1 while mapped                             */
     const uint8_t* pool;    /* the cache's frame pool (one hop for links) */
-    uint64_t pad_;
+    uint32_t prot;          /* PROT_READ | PROT_WRITE                     */
+    uint32_t pad_;
 };
 
 /* Cache descriptor, one copy in device memory per ap_cache_t. */
@@ -233,6 +243,20 @@ template <> __device__ __forceinline__ double ld_data<double>(const double* p) {
     return __ldcg(p);
 }
 
+template <class T> __device__ __forceinline__ void st_data(T* p, const T& v);
+template <> __device__ __forceinline__ void st_data<uint32_t>(uint32_t* p, const uint32_t& v) {
+    __stcg(p, v);
+}
+template <> __device__ __forceinline__ void st_data<unsigned long long>(unsigned long long* p,
+                                                                        const unsigned long long& v) {
+    __stcg(p, v);
+}
+template <> __device__ __forceinline__ void st_data<uint4>(uint4* p, const uint4& v) { __stcg(p, v); }
+template <> __device__ __forceinline__ void st_data<int32_t>(int32_t* p, const int32_t& v) {
+    __stcg(p, v);
+}
+template <> __device__ __forceinline__ void st_data<float>(float* p, const float& v) { __stcg(p, v); }
+
 __device__ __forceinline__ void set_err(const dev_cache* c, int code) {
     atomicCAS(c->err, 0, code);
 }
@@ -259,9 +283,43 @@ static __device__ AP_SLOW_ATTR void unlink_lanes(unsigned m, bool mine, const de
     unsigned lane = lane_id();
     if (mine && lane == (unsigned)(__ffs(grp) - 1)) {
         unsigned n = __popc(grp);
+#ifdef AP_DEBUG
+        printf("[unlink] w%u m%08x grp%08x n%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, grp, n, (unsigned long long)page);
+#endif
         red_add_release(r->pte + page, (uint64_t)0 - (uint64_t)n);
         stat_add(&my_stats(r->cache)->unlinks, 1);
     }
+}
+
+/* -------------------------------------------------------------------------
+ * Write-back (writable mappings, NEXT N3): the lanes in m copy frame f to
+ * the page's bytes in host memory over the host link (zero-copy 16-B
+ * stores), then fence at system scope so the host sees them before the page
+ * can be refilled from it. */
+__device__ __forceinline__ void writeback_page(unsigned m, const dev_cache* c, const dev_region* r,
+                                               uint64_t f, uint64_t pg) {
+    const unsigned lane = __popc(m & lanemask_lt());
+    const unsigned nl = __popc(m);
+    const uint64_t P = 1ull << c->log2_page;
+    const uint8_t* src = c->pool + f * P;
+    uint8_t* dst = const_cast<uint8_t*>(r->host) + pg * P;
+    const uint64_t avail = r->bytes - pg * P;
+    const uint64_t len = avail < P ? avail : P;
+    const uint64_t nvec = len / 16;
+    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    uint4* d4 = reinterpret_cast<uint4*>(dst);
+    constexpr int U = 8;
+    uint64_t i = lane;
+    for (; i + (uint64_t)nl * (U - 1) < nvec; i += (uint64_t)nl * U) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = __ldcg(s4 + i + (uint64_t)nl * u);
+#pragma unroll
+        for (int u = 0; u < U; ++u) __stcs(d4 + i + (uint64_t)nl * u, v[u]);
+    }
+    for (; i < nvec; i += nl) __stcs(d4 + i, __ldcg(s4 + i));
+    for (uint64_t b = nvec * 16 + lane; b < len; b += nl) dst[b] = src[b];
+    __threadfence_system();
 }
 
 /* -------------------------------------------------------------------------
@@ -293,18 +351,21 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         }
     }
     unsigned still = __ballot_sync(m, want && !got);
-    /* at most two laps of the clock per attempt (second chance), then back off */
-    const uint64_t lap = (c->frames + 31) / 32;
+    /* the lanes present (possibly fewer than 32) each examine one frame per
+     * clock step; at most two laps per attempt (second chance), then back off */
+    const unsigned nl = __popc(m);
+    const unsigned rk = __popc(m & lanemask_lt());
+    const uint64_t lap = (c->frames + nl - 1) / nl;
     uint32_t steps = c->sweep_steps < 2 * lap + 1 ? c->sweep_steps : (uint32_t)(2 * lap + 1);
     unsigned long long evicted = 0;
     while (still && steps--) {
         unsigned long long hb = 0;
         if ((int)lane == first)
-            hb = fetch_add_relaxed(c->clock_hand, c->policy == POLICY_CLOCK ? 32ull : 1ull);
+            hb = fetch_add_relaxed(c->clock_hand, c->policy == POLICY_CLOCK ? (unsigned long long)nl : 1ull);
         hb = __shfl_sync(m, hb, first);
         uint64_t f;
-        if (c->policy == POLICY_CLOCK) f = (hb + lane) % c->frames;
-        else f = sm64(c->policy_seed ^ (hb << 5) ^ lane) % c->frames;
+        if (c->policy == POLICY_CLOCK) f = (hb + rk) % c->frames;
+        else f = sm64(c->policy_seed ^ (hb << 5) ^ rk) % c->frames;
         bool elig = false;
         uint64_t e = 0;
         uint64_t* q = nullptr;
@@ -321,8 +382,22 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         const unsigned cand = __ballot_sync(m, elig);
         const int need_n = __popc(still);
         bool won = false;
-        if (elig && __popc(cand & lanemask_lt()) < need_n) won = (cas_acquire(q, e, PTE_EMPTY) == e);
+        /* a dirty victim is claimed into LOADING (faulters wait) until its
+         * bytes are back in the file, then released to EMPTY */
+        if (elig && __popc(cand & lanemask_lt()) < need_n)
+            won = (cas_acquire(q, e, (e & PTE_DIRTY) ? PTE_LOADING : PTE_EMPTY) == e);
         const unsigned wonm = __ballot_sync(m, won);
+        unsigned dirtym = __ballot_sync(m, won && (e & PTE_DIRTY));
+        while (dirtym) {
+            const int L = __ffs(dirtym) - 1;
+            dirtym &= dirtym - 1;
+            const unsigned long long vown = __shfl_sync(m, (unsigned long long)own, L);
+            const uint64_t vf = __shfl_sync(m, (unsigned long long)f, L);
+            const dev_region* vr = c->regions + ((vown >> 48) - 1);
+            writeback_page(m, c, vr, vf, vown & PAGE_MASK48);
+            __syncwarp(m);
+            if ((int)lane == L) red_add_release(q, (uint64_t)0 - PTE_LOADING);
+        }
         const int nwon = __popc(wonm);
         evicted += nwon;
         const bool mine_still = (still >> lane) & 1u;
@@ -339,6 +414,16 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         stat_add(&my_stats(c)->evictions, evicted);
         if (still) stat_add(&my_stats(c)->nofree, 1);
     }
+#ifdef AP_DEBUG
+    if (still && (int)lane == first) {
+        const uint64_t own0 = ld_relaxed(c->owner);
+        const uint64_t e0 = own0 ? ld_relaxed(c->regions[(own0 >> 48) - 1].pte + (own0 & PAGE_MASK48)) : 0;
+        if ((clock64() & 0xfffff) < 200)
+            printf("[nofree] sm %u warp %u m %08x own0 %llx e0 %llx hand %llu\n", sm_id(),
+                   (unsigned)(threadIdx.x >> 5), m, (unsigned long long)own0, (unsigned long long)e0,
+                   (unsigned long long)*c->clock_hand);
+    }
+#endif
     return got;
 }
 
@@ -435,6 +520,9 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
          * counts on non-VALID entries: publish and revert are adds, claims
          * are CASes from exactly EMPTY (R-A17). */
         uint64_t old = is_leader ? add_acquire(pte, n) : 0;
+#ifdef AP_DEBUG
+        if (is_leader && (old >> 62) == 2) printf("[link] w%u m%08x n%u pg %llu old %llx\n", (unsigned)(threadIdx.x >> 5), m, n, (unsigned long long)pg, (unsigned long long)old);
+#endif
         if (is_leader) {
             if ((old >> 62) == 2) {
                 st = ST_LINKED;
@@ -494,6 +582,9 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             }
             fence_gpu();
             __syncwarp(m);
+#ifdef AP_DEBUG
+            if ((int)lane == L) printf("[publish] w%u m%08x n%u f%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, n, f, (unsigned long long)fpg);
+#endif
             if ((int)lane == L)
                 red_add_release(pte, (PTE_VALID - PTE_LOADING) | PTE_REF | ((uint64_t)f << 32) |
                                          (uint64_t)n);
@@ -647,6 +738,84 @@ __device__ AP_SLOW_ATTR tile_out<T, N> read_tile_slow(unsigned m, uint64_t x, ui
     return t;
 }
 
+/* Store path (writable mappings, NEXT N3; Fig. 3's `*ptr = 25`, PAPER.md:
+ * 134): every lane in m stores v at its offset.  Linked lanes store first;
+ * then, if some lanes must fault while frames are scarce, the warp drops
+ * every link it holds; then unlinked lanes are handled one page group at a
+ * time: linked through the fault path (one page, so the group
+ * comes back linked), the page marked DIRTY once (leader OR; the pointer
+ * remembers it in XL_DIRTY), the lanes store, and under pressure the group
+ * unlinks again if other groups are still waiting -- a warp never waits for
+ * a frame while pinning one (R-A19).  Returns the new translation. */
+template <class T>
+__device__ AP_SLOW_ATTR slow_out<T> store_slow(unsigned m, uint64_t x, uint64_t page,
+                                               const dev_region* r, T v) {
+    const dev_cache* c = r->cache;
+    const uint32_t lg = c->log2_page;
+    if (!(r->prot & PROT_WRITE)) {
+        set_err(c, ERR_PERM);
+        return slow_out<T>{x, page, T{}};
+    }
+    const unsigned lane = lane_id();
+    /* 1. lanes already linked store through their link (marking the page
+     *    DIRTY once per page if this link has not yet) */
+    const bool lnk = (x >> 63) != 0;
+    bool done = false;
+    {
+        const bool mark = lnk && !(x & XL_DIRTY);
+        const unsigned long long key = mark ? (((unsigned long long)r->id << 48) | page) : ~0ull;
+        const unsigned grp = __match_any_sync(m, key);
+        if (mark && (int)lane == __ffs(grp) - 1) red_or_relaxed(r->pte + page, PTE_DIRTY);
+        if (lnk) {
+            x |= XL_DIRTY;
+            st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
+            done = true;
+        }
+    }
+    /* 2. before any lane faults under frame pressure, the warp drops the
+     *    links it holds (the values are stored), so it never waits for a
+     *    frame while pinning one (R-A19) */
+    const bool pressure = *(volatile unsigned long long*)c->free_head >= c->nfree;
+    if (pressure && __any_sync(m, !done) && __any_sync(m, lnk)) {
+        unlink_lanes(m, lnk, r, page);
+        if (lnk) x = (page << lg) | (x & ((1ull << lg) - 1));
+    }
+    /* 3. unlinked lanes, one page group at a time */
+    for (;;) {
+        const unsigned pend = __ballot_sync(m, !done);
+        if (!pend) break;
+        const int L = __ffs(pend) - 1;
+        const uint64_t mypg = x >> lg;
+        const uint64_t lpg = __shfl_sync(m, mypg, L);
+        const unsigned long long lr = __shfl_sync(m, (unsigned long long)r, L);
+        const bool in = !done && mypg == lpg && (unsigned long long)r == lr;
+        const unsigned mg = __ballot_sync(m, in);
+        if (in) {
+            const slow_out<T> o = deref_slow<T>(mg, x, page, r);
+            x = o.x;
+            page = o.page;
+            const bool ok = (x >> 63) != 0;
+            const unsigned okm = __ballot_sync(mg, ok);
+            if (ok && (int)lane == __ffs(okm) - 1) red_or_relaxed(r->pte + page, PTE_DIRTY);
+            if (ok) {
+                x |= XL_DIRTY;
+                st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
+            }
+            /* pressure re-read: this group may have taken the last free frame */
+            const bool now_pressure = *(volatile unsigned long long*)c->free_head >= c->nfree;
+            const bool drop = ok && now_pressure && __popc(pend) > __popc(mg);
+            if (__any_sync(mg, drop)) {
+                unlink_lanes(mg, drop, r, page);
+                if (drop) x = (page << lg) | (x & ((1ull << lg) - 1));
+            }
+            /* a lane the fault path could not link (watchdog) drops its store */
+            done = true;
+        }
+        __syncwarp(m);
+    }
+    return slow_out<T>{x, page, T{}};
+}
+
 }  // namespace detail
 
 /* ======================================================================
@@ -709,6 +878,19 @@ struct ptr {
         x = o.x;
         page = o.page;
         return o.val;
+    }
+
+    /* Store through the pointer (writable mappings; Fig. 3 `*ptr = 25`). */
+    __device__ __forceinline__ void store(const T& v) {
+        const unsigned m = __activemask();
+        const bool ok = (x & (XL_VALID | XL_DIRTY)) == (XL_VALID | XL_DIRTY);
+        if (__all_sync(m, ok)) {
+            detail::st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
+            return;
+        }
+        const detail::slow_out<T> o = detail::store_slow<T>(m, x, page, r, v);
+        x = o.x;
+        page = o.page;
     }
 
     /* p[i] without moving p: a linked lane whose target stays in the page
@@ -808,6 +990,14 @@ struct ptr {
         ptr q(*this);
         q.x += (uint64_t)(d * (int64_t)sizeof(T));
         return q;
+    }
+
+    /* True when the cache's free list is exhausted (frames are recycled by
+     * eviction).  A thread that holds one linked pointer while another one
+     * may fault should release the first under pressure (R-A19). */
+    __device__ __forceinline__ bool cache_pressure() const {
+        const dev_cache* c = r->cache;
+        return *(volatile unsigned long long*)c->free_head >= c->nfree;
     }
 
     /* Unlink now (also done by the destructor and by assignment). */

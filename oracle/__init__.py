@@ -12,6 +12,10 @@ What it computes (citations are PAPER.md lines; readings R-Ax are DESIGN.md's):
   Pinned by tests/test_oracle_reads.py: the splitmix64 and FNV-1a-64 published
   test vectors, brute-force re-reads through numpy views on tiny files, and
   closed-form access-pattern properties (distinct pages per warp, coverage).
+* O1' writes -- the file with each stored element replaced (plain
+  indexing; Fig. 3 `*ptr = 25`).  Pinned by the published
+  splitmix vectors, coverage of the SEQ pattern and bijectivity of the
+  permutation pattern (tests/test_oracle_writes.py).
 * O2 fault-path invariants -- `invariants.py`.
   Pinned by negative tests: a dump that breaks each invariant is rejected.
 * O3 collage -- histogram -> LSH keys -> candidate buckets
@@ -62,6 +66,9 @@ def _load():
         lib.or_build_index.argtypes = [vp, u32, u64, u32, u32, vp, vp, i32, u32, vp, vp, ci]
         lib.or_ssd.restype = u32
         lib.or_ssd.argtypes = [vp, vp]
+        lib.or_perm_idx.restype = u64
+        lib.or_perm_idx.argtypes = [u64, u64]
+        lib.or_apply_writes.argtypes = [vp, u64, u32, ci, u64, u32, u64, u64]
         lib.or_collage.argtypes = [vp, u32, u32, u32, u32, u32, vp, vp, i32, vp, u32, u64,
                                    vp, vp, u64, u64, vp, ci]
         _lib = lib
@@ -118,6 +125,18 @@ def read_divergent(file: np.ndarray, nbytes, page, elem, nthreads, reads, seed, 
     _load().or_read_divergent(_p(file), nbytes, page, elem, nthreads, reads, seed, _p(ck),
                               threads or threads_default())
     return ck
+
+
+def perm_idx(k, M):
+    return int(_load().or_perm_idx(k, M))
+
+
+def apply_writes(file: np.ndarray, elem, pattern, nthreads=0, reads=0, span=None, seed=0):
+    """The file after the write benchmark's stores (a new array)."""
+    out = file.copy()
+    span = file.nbytes if span is None else span
+    _load().or_apply_writes(_p(out), file.nbytes, elem, pattern, nthreads, reads, span, seed)
+    return out
 
 
 # ---------------------------------------------------------------- O3 collage

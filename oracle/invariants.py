@@ -16,7 +16,7 @@ for its page cache:
 
 Dump format (the C-ABI's ap_cache_dump / ap_region_dump_pte, include/ap.h):
   pte[r]   uint64[npages_r]   bits 63:62 state (0 EMPTY, 1 LOADING, 2 VALID),
-                              bit 61 reference bit, bits 60:32 frame,
+                              bit 61 reference bit, bit 60 dirty, bits 59:32 frame,
                               bits 31:0 reference count
   owner    uint64[frames]     0 = none, else ((region+1) << 48) | page
   free_left int               frames still on the free list
@@ -30,7 +30,7 @@ def pte_fields(pte):
     pte = np.asarray(pte, dtype=np.uint64)
     state = (pte >> np.uint64(62)).astype(np.int64)
     ref = ((pte >> np.uint64(61)) & np.uint64(1)).astype(np.int64)
-    frame = ((pte >> np.uint64(32)) & np.uint64((1 << 29) - 1)).astype(np.int64)
+    frame = ((pte >> np.uint64(32)) & np.uint64((1 << 28) - 1)).astype(np.int64)
     rc = (pte & np.uint64(0xFFFFFFFF)).astype(np.int64)
     return state, ref, frame, rc
 

@@ -256,3 +256,62 @@ void or_collage(const uint8_t* img, uint32_t W, uint32_t H, uint32_t L, uint32_t
         winners[2 * k + 1] = best_dist;
     }
 }
+
+/* ------------------------------------------------------------------ */
+/* Writes (NEXT N3; Fig. 3 `*ptr = 25`): the file after the */
+/* benchmark's stores is the file with each stored element replaced --    */
+/* plain indexing again (a store through an apointer is a store to the    */
+/* file).  Workload definitions as DESIGN.md / include/ap.h.              */
+/* ------------------------------------------------------------------ */
+static void or_wval(uint64_t seed, uint64_t e, uint32_t elem, uint8_t* out) {
+    if (elem == 4) {
+        uint32_t v = (uint32_t)or_sm64_(seed ^ e);
+        memcpy(out, &v, 4);
+    } else if (elem == 8) {
+        uint64_t v = or_sm64_(seed ^ e);
+        memcpy(out, &v, 8);
+    } else {
+        uint64_t a = or_sm64_(seed ^ (2 * e)), b = or_sm64_(seed ^ (2 * e + 1));
+        memcpy(out, &a, 8);
+        memcpy(out + 8, &b, 8);
+    }
+}
+
+static uint64_t or_gcd(uint64_t a, uint64_t b) {
+    while (b) {
+        uint64_t t = a % b;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+
+/* the permutation's multiplier: largest odd a <= floor(M * 0.618...) (the
+ * golden-ratio fraction 0x9E3779B97F4A7C15 / 2^64), stepped up by 2 until
+ * gcd(a, M) = 1; element k of the write sequence goes to k*a mod M. */
+uint64_t or_perm_mult(uint64_t M) {
+    uint64_t a = (uint64_t)(((unsigned __int128)M * 0x9E3779B97F4A7C15ull) >> 64) | 1;
+    if (a >= M) a = 1;
+    while (or_gcd(a, M) != 1) a += 2;
+    return a % M;
+}
+
+uint64_t or_perm_idx(uint64_t k, uint64_t M) {
+    unsigned __int128 A = or_perm_mult(M);
+    return (uint64_t)(((unsigned __int128)(k % M) * A) % M);
+}
+
+/* pattern 0 (SEQ): every whole element of [0, span); pattern 1 (UNIFORM):
+ * element or_perm_idx(t*reads + i, bytes/elem) for t < nthreads, i < reads. */
+void or_apply_writes(uint8_t* buf, uint64_t bytes, uint32_t elem, int pattern, uint64_t nthreads,
+                     uint32_t reads, uint64_t span, uint64_t seed) {
+    if (pattern == 0) {
+        for (uint64_t e = 0; (e + 1) * elem <= span; ++e) or_wval(seed, e, elem, buf + e * elem);
+    } else {
+        uint64_t M = bytes / elem;
+        for (uint64_t k = 0; k < nthreads * (uint64_t)reads; ++k) {
+            uint64_t e = or_perm_idx(k, M);
+            or_wval(seed, e, elem, buf + e * elem);
+        }
+    }
+}

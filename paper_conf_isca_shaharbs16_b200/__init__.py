@@ -9,7 +9,7 @@ import ctypes
 import numpy as np
 
 from . import _lib
-from ._lib import (AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_TILE, AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK,  # noqa: F401
+from ._lib import (AP_PROT_READ, AP_PROT_WRITE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_TILE, AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK,  # noqa: F401
                    AP_POLICY_RANDOM, AP_SEQ, AP_UNIFORM, APError, ap_bench_cfg, ap_collage_in,
                    ap_stats_t)
 
@@ -77,6 +77,18 @@ def ap_mmap(cache, host_buf, nbytes=None):
     nbytes = _nbytes(host_buf) if nbytes is None else nbytes
     _lib.check("ap_mmap", _lib.lib().ap_mmap(cache, _ptr(host_buf), nbytes, ctypes.byref(r)))
     return r.value
+
+
+def ap_mmap_prot(cache, host_buf, prot, nbytes=None):
+    r = ctypes.c_uint32()
+    nbytes = _nbytes(host_buf) if nbytes is None else nbytes
+    _lib.check("ap_mmap_prot", _lib.lib().ap_mmap_prot(cache, _ptr(host_buf), nbytes, prot,
+                                                       ctypes.byref(r)))
+    return r.value
+
+
+def ap_msync(cache, region):
+    _lib.check("ap_msync", _lib.lib().ap_msync(cache, region))
 
 
 def ap_munmap(cache, region):
@@ -149,6 +161,16 @@ def bench_cfg(pattern, elem_bytes, grid, block, reads_per_thread=0, passes=1, un
 def ap_bench_read(cache, region, cfg, out_dev, stream=None):
     _lib.check("ap_bench_read", _lib.lib().ap_bench_read(cache, region, ctypes.byref(cfg),
                                                          _ptr(out_dev), _stream(stream)))
+
+
+def ap_bench_write(cache, region, cfg, stream=None):
+    _lib.check("ap_bench_write", _lib.lib().ap_bench_write(cache, region, ctypes.byref(cfg),
+                                                           _stream(stream)))
+
+
+def ap_bench_copy(cache, src, dst, cfg, stream=None):
+    _lib.check("ap_bench_copy", _lib.lib().ap_bench_copy(cache, src, dst, ctypes.byref(cfg),
+                                                         _stream(stream)))
 
 
 def ap_bench_read_host(cache, region, cfg, out_host):

@@ -17,6 +17,8 @@ AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
 AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE = 0, 1, 2
 AP_SCHED_NATURAL, AP_SCHED_LSH = 0, 1
+AP_PROT_READ, AP_PROT_WRITE = 1, 2
+AP_EPERM = -9
 
 u64, u32, i32, vp, ci = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int
 
@@ -83,6 +85,10 @@ def lib():
                                         ctypes.POINTER(ctypes.c_double)]),
             "ap_collage_run": (ci, [vp, u32, ctypes.POINTER(ap_collage_in), vp, vp]),
             "ap_bench_latency": (ci, [vp, u32, ci, u32, ctypes.POINTER(u64)]),
+            "ap_mmap_prot": (ci, [vp, vp, u64, ci, ctypes.POINTER(u32)]),
+            "ap_msync": (ci, [vp, u32]),
+            "ap_bench_write": (ci, [vp, u32, ctypes.POINTER(ap_bench_cfg), vp]),
+            "ap_bench_copy": (ci, [vp, u32, u32, ctypes.POINTER(ap_bench_cfg), vp]),
             "ap_lsh_build_index": (ci, [vp, u32, u64, u32, u32, u32, u32, i32, vp, vp, vp, vp,
                                         vp]),
         }
@@ -99,7 +105,7 @@ EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", 
             "ap_cache_reset", "ap_cache_set_policy", "ap_cache_set_tuning",
             "ap_last_device_error", "ap_cache_dump", "ap_region_dump_pte", "ap_prefill",
             "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index",
-            "ap_bench_latency"]
+            "ap_bench_latency", "ap_mmap_prot", "ap_msync", "ap_bench_write", "ap_bench_copy"]
 
 
 def check(fn, rc):

@@ -448,3 +448,198 @@ extern "C" int ap_bench_latency(ap_cache_t c, ap_region_t region, int op, uint32
     cycles[1] = h[1];
     return AP_OK;
 }
+
+/* ------------------------------------------------------------------------
+ * Writes through apointers (NEXT N3; Fig. 3 `*ptr = 25`) and
+ * the apointer-to-apointer copy (the Table II copy kernel).
+ * Value written at element e: low bytes of sm64(seed ^ e) (16-B elements:
+ * sm64(seed ^ 2e), sm64(seed ^ (2e+1))).  Offsets: SEQ units as k_seq, or a
+ * race-free permutation e = (t*R + i) * a mod M (perm_mult). */
+namespace {
+
+template <class T> __device__ __forceinline__ T wval(uint64_t seed, uint64_t e);
+template <> __device__ __forceinline__ uint32_t wval<uint32_t>(uint64_t seed, uint64_t e) {
+    return (uint32_t)ap::detail::sm64(seed ^ e);
+}
+template <> __device__ __forceinline__ unsigned long long wval<unsigned long long>(uint64_t seed,
+                                                                                  uint64_t e) {
+    return ap::detail::sm64(seed ^ e);
+}
+template <> __device__ __forceinline__ uint4 wval<uint4>(uint64_t seed, uint64_t e) {
+    const uint64_t a = ap::detail::sm64(seed ^ (2 * e)), b = ap::detail::sm64(seed ^ (2 * e + 1));
+    return make_uint4((uint32_t)a, (uint32_t)(a >> 32), (uint32_t)b, (uint32_t)(b >> 32));
+}
+
+/* permutation multiplier: the odd number nearest below 0.618*M that is
+ * coprime with M (a bijection of [0, M) that scatters neighbours) */
+__host__ __device__ inline uint64_t gcd_u64(uint64_t a, uint64_t b) {
+    while (b) {
+        const uint64_t t = a % b;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+__host__ __device__ inline uint64_t perm_mult(uint64_t M) {
+    uint64_t a = (uint64_t)(((unsigned __int128)M * 0x9E3779B97F4A7C15ull) >> 64) | 1;
+    if (a >= M) a = 1;
+    while (gcd_u64(a, M) != 1) a += 2;
+    return a % M;
+}
+__device__ __forceinline__ uint64_t perm_idx(uint64_t k, uint64_t M, uint64_t A) {
+    return ((k % M) * A) % M;
+}
+
+template <class T, int PAT>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
+    k_write(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    if constexpr (PAT == AP_SEQ) {
+        const uint64_t w = t >> 5, lane = t & 31;
+        const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
+        const uint32_t per_unit = a.unit / (32 * E);
+        for (uint64_t u = w; u < nunits; u += W) {
+            const uint64_t e0 = u * (a.unit / E) + lane;
+            ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
+            for (uint32_t j = 0; j < per_unit; ++j) {
+                const uint64_t e = e0 + 32ull * j;
+                if ((e + 1) * E <= a.span) q.store(wval<T>(a.seed, e));
+                q += 32;
+            }
+        }
+    } else {
+        const uint64_t M = a.bytes / E;
+        const uint64_t A = perm_mult(M);
+        ap::ptr<T> p = ap::gvmmap<T>(c, region, 0);
+        uint64_t cur = 0;
+        for (uint32_t i = 0; i < a.reads; ++i) {
+            const uint64_t e = perm_idx(t * a.reads + i, M, A);
+            p += (int64_t)e - (int64_t)cur;
+            cur = e;
+            p.store(wval<T>(a.seed, e));
+        }
+    }
+}
+
+/* dst[e] = src[e] for e < span/E, both through apointers (the copy kernel
+ * of PAPER.md:312: tiled reads, stores one element at a time). */
+template <class T>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
+    k_copy(const ap::dev_cache* __restrict__ c, uint32_t src, uint32_t dst, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    constexpr int CT = 8;
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t w = t >> 5, lane = t & 31;
+    const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
+    const uint32_t per_unit = a.unit / (32 * E);
+    for (uint64_t u = w; u < nunits; u += W) {
+        const uint64_t e0 = u * (a.unit / E) + lane;
+        const bool whole = (u + 1) * a.unit <= a.span;
+        ap::ptr<T> s = ap::gvmmap<T>(c, src, e0 * E);
+        ap::ptr<T> d = ap::gvmmap<T>(c, dst, e0 * E);
+        uint32_t j = 0;
+        if (whole) {
+            for (; j + CT <= per_unit; j += CT) {
+                T v[CT];
+                s.read_tile(v, 32);
+                /* never hold the source pin while the destination may fault
+                 * on a recycled cache (R-A19) */
+                if (s.cache_pressure()) s.release();
+#pragma unroll
+                for (int k = 0; k < CT; ++k) {
+                    d.store(v[k]);
+                    d += 32;
+                }
+                if (d.cache_pressure()) d.release();
+                s += 32 * CT;
+            }
+        }
+        for (; j < per_unit; ++j) {
+            if ((e0 + 32ull * j + 1) * E <= a.span) {
+                const T v = *s;
+                if (s.cache_pressure()) s.release();
+                d.store(v);
+                if (d.cache_pressure()) d.release();
+            }
+            s += 32;
+            d += 32;
+        }
+    }
+}
+
+template <class T>
+cudaError_t launch_write(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg,
+                         const BenchArgs& a, cudaStream_t s) {
+    if (cfg->pattern == AP_SEQ)
+        k_write<T, AP_SEQ><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+    else
+        k_write<T, AP_UNIFORM><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+extern "C" int ap_bench_write(ap_cache_t c, ap_region_t region, const ap_bench_cfg* cfg,
+                              void* stream) {
+    if (!ap_region_ok(c, region) || !cfg) return AP_EINVAL;
+    if (!(c->reg[region].prot & AP_PROT_WRITE)) return AP_EINVAL;
+    const uint32_t E = cfg->elem_bytes;
+    if ((E != 4 && E != 8 && E != 16) || cfg->grid == 0 || cfg->block == 0 ||
+        cfg->block > AP_BENCH_THREADS || cfg->block % 32)
+        return AP_EINVAL;
+    BenchArgs a{};
+    a.bytes = c->reg[region].bytes;
+    a.span = cfg->span_bytes ? cfg->span_bytes : a.bytes;
+    a.unit = cfg->unit_bytes;
+    a.reads = cfg->reads_per_thread;
+    a.seed = cfg->seed;
+    if (cfg->pattern == AP_SEQ) {
+        if (a.unit == 0 || a.unit % (32 * E) || c->page % a.unit || a.span > a.bytes) return AP_EINVAL;
+    } else if (cfg->pattern == AP_UNIFORM) {
+        if ((uint64_t)cfg->grid * cfg->block * cfg->reads_per_thread > a.bytes / E) return AP_EINVAL;
+        if (a.bytes / E > (1ull << 32)) return AP_ERANGE; /* perm_idx products stay in 64 bits */
+    } else {
+        return AP_EINVAL;
+    }
+    ap_device_guard g(c->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    switch (E) {
+        case 4: e = launch_write<uint32_t>(c, region, cfg, a, s); break;
+        case 8: e = launch_write<unsigned long long>(c, region, cfg, a, s); break;
+        default: e = launch_write<uint4>(c, region, cfg, a, s);
+    }
+    AP_CUDA_TRY(e);
+    return AP_OK;
+}
+
+extern "C" int ap_bench_copy(ap_cache_t c, ap_region_t src, ap_region_t dst,
+                             const ap_bench_cfg* cfg, void* stream) {
+    if (!ap_region_ok(c, src) || !ap_region_ok(c, dst) || !cfg || src == dst) return AP_EINVAL;
+    if (!(c->reg[dst].prot & AP_PROT_WRITE)) return AP_EINVAL;
+    const uint32_t E = cfg->elem_bytes;
+    if ((E != 4 && E != 8 && E != 16) || cfg->grid == 0 || cfg->block == 0 ||
+        cfg->block > AP_BENCH_THREADS || cfg->block % 32)
+        return AP_EINVAL;
+    BenchArgs a{};
+    a.bytes = c->reg[src].bytes;
+    a.span = cfg->span_bytes ? cfg->span_bytes : a.bytes;
+    a.unit = cfg->unit_bytes;
+    if (a.unit == 0 || a.unit % (32 * E) || c->page % a.unit || a.span > a.bytes ||
+        a.span > c->reg[dst].bytes)
+        return AP_EINVAL;
+    ap_device_guard g(c->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    switch (E) {
+        case 4: k_copy<uint32_t><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a); break;
+        case 8:
+            k_copy<unsigned long long><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+            break;
+        default: k_copy<uint4><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+    }
+    AP_CUDA_TRY(cudaGetLastError());
+    return AP_OK;
+}

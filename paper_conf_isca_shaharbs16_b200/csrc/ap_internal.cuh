@@ -21,6 +21,7 @@ struct ap_region_host {
     uint64_t* pte = nullptr; /* device                                     */
     bool registered = false; /* we called cudaHostRegister                 */
     bool live = false;
+    uint32_t prot = 1;       /* AP_PROT_*                                  */
 };
 
 struct ap_cache_s {

@@ -29,6 +29,7 @@ extern "C" const char* ap_strerror(int code) {
         case AP_EFAULT: return "device: dereference outside the mapped region or misaligned";
         case AP_ENOFRAME: return "device: no evictable frame";
         case AP_ETIMEDOUT: return "device: fault-path watchdog expired";
+        case AP_EPERM: return "device: store through a read-only mapping";
         default: return "unknown error";
     }
 }
@@ -99,6 +100,23 @@ __global__ void k_prefill(const ap::dev_cache* __restrict__ c, uint32_t region, 
     }
 }
 
+/* msync: one warp per page; VALID + DIRTY pages are copied back to the
+ * file and marked clean (no kernel may run concurrently). */
+__global__ void k_writeback(const ap::dev_cache* __restrict__ c, uint32_t region) {
+    const ap::dev_region* r = c->regions + region;
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) / 32;
+    const uint64_t nwarps = (uint64_t)gridDim.x * blockDim.x / 32;
+    for (uint64_t p = warp; p < r->npages; p += nwarps) {
+        const uint64_t e = r->pte[p];
+        if ((e >> 62) == 2 && (e & ap::PTE_DIRTY)) {
+            ap::detail::writeback_page(0xffffffffu, c, r, (e >> 32) & ap::PTE_FRAME_MASK, p);
+            __syncwarp();
+            if ((threadIdx.x & 31) == 0)
+                atomicAnd((unsigned long long*)(r->pte + p), ~(unsigned long long)ap::PTE_DIRTY);
+        }
+    }
+}
+
 static int scan_refs(ap_cache_s* c, const ap_region_host& rg, int* result) {
     int* d_flag = nullptr;
     AP_CUDA_TRY(cudaMalloc(&d_flag, sizeof(int)));
@@ -129,7 +147,7 @@ static int rebuild_free_list(ap_cache_s* c) {
 
 /* ------------------------------------------------------------ the cache */
 extern "C" int ap_cache_create(uint64_t frames, uint32_t page_size, int device, ap_cache_t* out) {
-    if (!out || frames == 0 || frames > ap::PTE_FRAME_MASK) return AP_EINVAL;
+    if (!out || frames == 0 || frames > ap::PTE_FRAME_MASK) return AP_EINVAL; /* < 2^28 */
     if (page_size < 4096 || page_size > (2u << 20) || (page_size & (page_size - 1))) return AP_EINVAL;
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return AP_EINVAL;
@@ -216,7 +234,13 @@ extern "C" int ap_cache_destroy(ap_cache_t c) {
 
 /* ------------------------------------------------------------ regions */
 extern "C" int ap_mmap(ap_cache_t c, const void* host_buf, uint64_t bytes, ap_region_t* out) {
+    return ap_mmap_prot(c, host_buf, bytes, AP_PROT_READ, out);
+}
+
+extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, int prot,
+                            ap_region_t* out) {
     if (!c || !host_buf || bytes == 0 || !out) return AP_EINVAL;
+    if (!(prot & AP_PROT_READ) || (prot & ~(AP_PROT_READ | AP_PROT_WRITE))) return AP_EINVAL;
     if (((uintptr_t)host_buf) & 15) return AP_EINVAL;
     const uint64_t npages = (bytes + c->page - 1) >> c->log2_page;
     if (npages >= (1ull << 48) || bytes >= (1ull << 60)) return AP_ERANGE;
@@ -238,7 +262,8 @@ extern "C" int ap_mmap(ap_cache_t c, const void* host_buf, uint64_t bytes, ap_re
     } else {
         unsigned flags = cudaHostRegisterMapped | cudaHostRegisterPortable;
         int ro = 0;
-        cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->device);
+        if (!(prot & AP_PROT_WRITE))
+            cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->device);
         if (ro) flags |= cudaHostRegisterReadOnly;
         e = cudaHostRegister(const_cast<void*>(host_buf), bytes, flags);
         if (e != cudaSuccess && ro) {
@@ -271,13 +296,26 @@ extern "C" int ap_mmap(ap_cache_t c, const void* host_buf, uint64_t bytes, ap_re
     d.pte = rg.pte;
     d.cache = c->d_cache;
     d.pool = c->pool;
+    d.prot = (uint32_t)prot;
     d.id = id;
     d.live = 1;
     AP_CUDA_TRY(cudaMemcpy(c->regions + id, &d, sizeof d, cudaMemcpyHostToDevice));
     rg.live = true;
+    rg.prot = (uint32_t)prot;
     if (id == c->reg.size()) c->reg.push_back(rg);
     else c->reg[id] = rg;
     *out = id;
+    return AP_OK;
+}
+
+extern "C" int ap_msync(ap_cache_t c, ap_region_t r) {
+    if (!ap_region_ok(c, r)) return AP_EINVAL;
+    if (!(c->reg[r].prot & AP_PROT_WRITE)) return AP_OK;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    k_writeback<<<c->num_sms * 4, 256>>>(c->d_cache, r);
+    AP_CUDA_TRY(cudaGetLastError());
+    AP_CUDA_TRY(cudaDeviceSynchronize());
     return AP_OK;
 }
 
@@ -285,6 +323,10 @@ extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
     if (!ap_region_ok(c, r)) return AP_EINVAL;
     ap_device_guard g(c->device);
     AP_CUDA_TRY(cudaDeviceSynchronize());
+    if (c->reg[r].prot & AP_PROT_WRITE) {
+        int rc0 = ap_msync(c, r);
+        if (rc0) return rc0;
+    }
     ap_region_host& rg = c->reg[r];
     int flag = 0;
     int rc = scan_refs(c, rg, &flag);
@@ -348,6 +390,11 @@ extern "C" int ap_cache_reset(ap_cache_t c) {
         if (rc) return rc;
         if (flag) return AP_EBUSY;
     }
+    for (uint32_t i = 0; i < c->reg.size(); ++i)
+        if (c->reg[i].live && (c->reg[i].prot & AP_PROT_WRITE)) {
+            int rc = ap_msync(c, i); /* dirty pages reach the file before eviction */
+            if (rc) return rc;
+        }
     for (auto& rg : c->reg)
         if (rg.live) AP_CUDA_TRY(cudaMemset(rg.pte, 0, rg.npages * 8));
     AP_CUDA_TRY(cudaMemset(c->owner, 0, c->frames * 8));

@@ -100,5 +100,27 @@ for g in (1, 4):
 check("unaligned invariants", check_invariants(ap, c, [r], 6) == [])
 ap.ap_munmap(c, r)
 ap.ap_cache_destroy(c)
+# writable mappings: scattered stores with 3 frames (dirty write-back during
+# the kernel), apointer-to-apointer copy with 4 frames
+fw = make_file(1 << 20, 9)
+want_w = oracle.apply_writes(fw, 4, 1, nthreads=256, reads=4, seed=3)
+c = ap.ap_cache_create(3, 4096)
+r = ap.ap_mmap_prot(c, fw, 3)
+ap.ap_bench_write(c, r, ap.bench_cfg(ap.AP_UNIFORM, 4, 2, 128, reads_per_thread=4, seed=3))
+torch.cuda.synchronize()
+check("writes device error", ap.ap_last_device_error(c) == 0)
+ap.ap_munmap(c, r)
+check("writes reach the file", np.array_equal(fw, want_w))
+src, dst = make_file(1 << 19, 10), make_file(1 << 19, 11)
+r1 = ap.ap_mmap(c, src)
+r2 = ap.ap_mmap_prot(c, dst, 3)
+ap.ap_bench_copy(c, r1, r2, ap.bench_cfg(ap.AP_SEQ, 16, 2, 64, unit_bytes=4096))
+torch.cuda.synchronize()
+check("copy device error", ap.ap_last_device_error(c) == 0)
+check("copy invariants", check_invariants(ap, c, [r1, r2], 3) == [])
+ap.ap_munmap(c, r2)
+ap.ap_munmap(c, r1)
+check("copy reaches the file", np.array_equal(dst, src))
+ap.ap_cache_destroy(c)
 print("ALL OK" if ok else "FAILURES")
 sys.exit(0 if ok else 1)
