@@ -893,6 +893,35 @@ struct ptr {
         page = o.page;
     }
 
+    /* Tiled store: p[k * stride] = v[k] for k < N, p unchanged.  One check
+     * for the tile when every lane is linked, its page already marked dirty
+     * and the tile inside the page; otherwise element by element. */
+    template <int N>
+    __device__ __forceinline__ void write_tile(const T (&v)[N], int64_t stride) {
+        const unsigned m = __activemask();
+        const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
+        const bool ok = (x & (XL_VALID | XL_DIRTY)) == (XL_VALID | XL_DIRTY) &&
+                        ((x ^ (x + span)) >> lg) == 0;
+        if (__all_sync(m, ok)) {
+            T* a = reinterpret_cast<T*>(x & XL_ADDR);
+#pragma unroll
+            for (int k = 0; k < N; ++k) detail::st_data<T>(a + k * stride, v[k]);
+            return;
+        }
+#pragma unroll 1
+        for (int k = 0; k < N; ++k) {
+            store(v[k]);
+            *this += stride;
+        }
+        *this -= N * stride;
+    }
+
+    /* warp-wide: every active lane is linked (and, for stores, marked dirty) */
+    __device__ __forceinline__ bool linked_all() const { return __all_sync(__activemask(), linked()); }
+    __device__ __forceinline__ bool store_ready() const {
+        return __all_sync(__activemask(), (x & (XL_VALID | XL_DIRTY)) == (XL_VALID | XL_DIRTY));
+    }
+
     /* p[i] without moving p: a linked lane whose target stays in the page
      * reads directly; otherwise a temporary pointer takes the fault. */
     __device__ __forceinline__ T operator[](int64_t i) {

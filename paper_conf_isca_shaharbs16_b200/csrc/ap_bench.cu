@@ -529,7 +529,7 @@ template <class T>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
     k_copy(const ap::dev_cache* __restrict__ c, uint32_t src, uint32_t dst, const BenchArgs a) {
     constexpr uint32_t E = sizeof(T);
-    constexpr int CT = 8;
+    constexpr int CT = TILE;
     const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     const uint64_t w = t >> 5, lane = t & 31;
     const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
@@ -544,17 +544,14 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
         if (whole) {
             for (; j + CT <= per_unit; j += CT) {
                 T v[CT];
+                /* never hold one pin while the other pointer faults on a
+                 * recycled cache (R-A19): drop it first under pressure */
+                if (!s.linked_all() && d.cache_pressure()) d.release();
                 s.read_tile(v, 32);
-                /* never hold the source pin while the destination may fault
-                 * on a recycled cache (R-A19) */
-                if (s.cache_pressure()) s.release();
-#pragma unroll
-                for (int k = 0; k < CT; ++k) {
-                    d.store(v[k]);
-                    d += 32;
-                }
-                if (d.cache_pressure()) d.release();
+                if (!d.store_ready() && s.cache_pressure()) s.release();
+                d.write_tile(v, 32);
                 s += 32 * CT;
+                d += 32 * CT;
             }
         }
         for (; j < per_unit; ++j) {
