@@ -439,12 +439,20 @@ def main():
         return
     import torch
     rank, local, world = env_rank()
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # AP_BENCH_SHARE_GPU=1 (validation only): every rank on cuda:0 with gloo
+    # collectives, to exercise the N>1 code paths on a one-GPU box.  Timings
+    # from such a run are not bench numbers.
+    share = os.environ.get("AP_BENCH_SHARE_GPU") == "1"
+    local_dev = 0 if share else local
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     if args.workload in ("c4", "c5"):
         import bench_collage
         res = bench_collage.run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler,

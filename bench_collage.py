@@ -190,6 +190,22 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
                is_copy=is_copy, src=src, cands=cands)
     # parity sample vs the oracle (rank 0): all blocks for c4, a sample for c5
     res["parity"] = None
+    # the gathered answer (N > 1): every rank's range arrives on rank 0
+    full = mgpu.gather_winners(win, rank, world, dist, nb) if world > 1 else None
+    if rank == 0 and full is not None and not args.no_cpu_baseline:
+        import oracle
+        fw = full.cpu().numpy().view(np.uint32)
+        o_off = off.cpu().numpy().view(np.uint32)
+        o_ids = ids.cpu().numpy().view(np.uint32)
+        ok = True
+        for r_ in range(world):  # 16 blocks from the start of every rank's range
+            rb0, rb1 = mgpu.block_range(nb, r_, world)
+            k = min(16, rb1 - rb0)
+            want = oracle.collage(img, proj, bias, cfg["w"], cfg["bb"], recs, cfg["stride"],
+                                  cfg["N"], o_off, o_ids, b0=rb0, nb=k,
+                                  threads=os.cpu_count() or 1)
+            ok = ok and bool(np.array_equal(want, fw[rb0:rb0 + k]))
+        res["gathered_parity"] = dict(ranks=world, blocks_per_rank=16, equal=ok)
     if rank == 0 and not args.no_cpu_baseline:
         import oracle
         o_off = off.cpu().numpy().view(np.uint32)
@@ -271,6 +287,8 @@ def emit_collage(args, res_all, world, METRIC):
         line["collage"]["apointer_warm_cache_s"] = round(r0["raw"]["warm_s"], 6)
         line["collage"]["overhead_warm_vs_raw"] = round(r0["raw"]["warm_s"] / r0["raw"]["raw_s"] - 1, 4)
         line["collage"]["raw_twin_equal"] = r0["raw"]["equal"]
+    if r0.get("gathered_parity"):
+        line["collage"]["gathered_parity_vs_oracle"] = r0["gathered_parity"]
     if r0["parity"]:
         p = r0["parity"]
         line["collage"]["parity_vs_oracle"] = {k: v for k, v in p.items() if k != "cpu_s"}

@@ -18,8 +18,10 @@ def gather_winners(win, rank, world, dist, nblocks, dst=0):
     if world == 1:
         return win
     rows = -(-nblocks // world)
-    pad = torch.full((rows, 2), -1, dtype=win.dtype, device=win.device)
-    pad[:win.shape[0]] = win
+    # gloo gathers host tensors; NCCL gathers device tensors over NVLink
+    dev = win.device if dist.get_backend() == "nccl" else "cpu"
+    pad = torch.full((rows, 2), -1, dtype=win.dtype, device=dev)
+    pad[:win.shape[0]] = win.to(dev)
     bufs = [torch.empty_like(pad) for _ in range(world)] if rank == dst else None
     dist.gather(pad, bufs, dst=dst)
     if rank != dst:
