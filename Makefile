@@ -18,10 +18,10 @@ CU_HDRS := $(wildcard $(CSRC)/*.cuh) $(wildcard include/*.h) $(wildcard include/
 all: synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so
 
 synth/libsynth.so: synth/synth.c
-	$(HOSTCC) $(CFLAGS) -shared $< -o $@
+	$(HOSTCC) $(CFLAGS) -shared $< -o $@ -lm
 
 oracle/liboracle.so: oracle/oracle.c
-	$(HOSTCC) $(CFLAGS) -shared $< -o $@
+	$(HOSTCC) $(CFLAGS) -shared $< -o $@ -lm
 
 $(PKG)/libapointer.so: $(CU_SRCS) $(CU_HDRS)
 	$(NVCC) $(NVFLAGS) -shared $(CU_SRCS) -o $@ -lcuda

@@ -223,6 +223,29 @@ int ap_bench_write(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg
 int ap_bench_copy(ap_cache_t cache, ap_region_t src, ap_region_t dst, const ap_bench_cfg* cfg,
                   void* stream);
 
+/* ap_bench_compute — the compute-intensity workloads of PAPER.md:332-359
+ * (Fig. 6a/6b; NEXT N4), apointer version or raw twin (mode).
+ *   work   0 ADD (acc += a[i] + b[i], b = a + span), 1 READ, 2 RANDOM-N (LCG
+ *          x = x*1664525 + 1013904223 iterated `iters` times), 3 REDUCE (warp
+ *          sum by shuffles), 4 FFT (32-point complex FFT across the warp,
+ *          re/im = low/high 16 bits, acc += trunc(|X|^2 / 65536)), 5 BITONIC
+ *          (warp bitonic sort, acc += sorted * (lane + 1));
+ *   elem_bytes 4 or 16 (a 16-B load feeds four independent word lanes);
+ *   span_bytes per vector, a multiple of the page size; warp w reads pages
+ *          w, w+W, ... one 4/16-B access at a time (`*q; q += 32`);
+ * out_dev: uint64[grid*block] per-thread accumulators.  Asynchronous. */
+typedef struct {
+    int32_t work;
+    uint32_t elem_bytes;
+    uint32_t grid, block;
+    uint32_t iters;
+    uint64_t span_bytes;
+    int32_t mode;
+    const void* raw_base;
+} ap_compute_cfg;
+int ap_bench_compute(ap_cache_t cache, ap_region_t region, const ap_compute_cfg* cfg,
+                     uint64_t* out_dev, void* stream);
+
 /* ap_bench_latency — Table I analogue: one warp, all
  * lanes on one (prefilled) page, coalesced 4-B accesses; op = 0 raw read,
  * 1 apointer read, 2 raw increment, 3 apointer increment, 4 raw read+inc,

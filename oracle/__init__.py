@@ -16,6 +16,11 @@ What it computes (citations are PAPER.md lines; readings R-Ax are DESIGN.md's):
   indexing; Fig. 3 `*ptr = 25`).  Pinned by the published
   splitmix vectors, coverage of the SEQ pattern and bijectivity of the
   permutation pattern (tests/test_oracle_writes.py).
+* compute workloads (Fig. 6) -- Add/Read/Random-N/Reduce/
+  FFT/Bitonic accumulators from their definitions (FFT as the O(n^2) DFT in
+  float64).  Pinned by closed forms in tests/test_oracle_compute.py (a
+  constant vector's DFT is an impulse, sorted input is a fixed point of the
+  sort, the LCG's published first step).
 * O2 fault-path invariants -- `invariants.py`.
   Pinned by negative tests: a dump that breaks each invariant is rejected.
 * O3 collage -- histogram -> LSH keys -> candidate buckets
@@ -69,6 +74,7 @@ def _load():
         lib.or_perm_idx.restype = u64
         lib.or_perm_idx.argtypes = [u64, u64]
         lib.or_apply_writes.argtypes = [vp, u64, u32, ci, u64, u32, u64, u64]
+        lib.or_compute.argtypes = [vp, u64, u32, u32, u64, ci, u32, vp, ci]
         lib.or_collage.argtypes = [vp, u32, u32, u32, u32, u32, vp, vp, i32, vp, u32, u64,
                                    vp, vp, u64, u64, vp, ci]
         _lib = lib
@@ -137,6 +143,14 @@ def apply_writes(file: np.ndarray, elem, pattern, nthreads=0, reads=0, span=None
     span = file.nbytes if span is None else span
     _load().or_apply_writes(_p(out), file.nbytes, elem, pattern, nthreads, reads, span, seed)
     return out
+
+
+def compute(file: np.ndarray, span, unit, elem, nthreads, work, iters=0, threads=None):
+    """Per-thread accumulators of the compute-intensity workloads (float64)."""
+    acc = np.empty(nthreads, dtype=np.float64)
+    _load().or_compute(_p(file), span, unit, elem, nthreads, work, iters, _p(acc),
+                       threads or threads_default())
+    return acc
 
 
 # ---------------------------------------------------------------- O3 collage

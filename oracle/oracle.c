@@ -315,3 +315,84 @@ void or_apply_writes(uint8_t* buf, uint64_t bytes, uint32_t elem, int pattern, u
         }
     }
 }
+
+/* ------------------------------------------------------------------ */
+/* Compute-intensity workloads (Fig. 6; NEXT N4): the */
+/* per-thread accumulators of ap_bench_compute, from their definitions:  */
+/* warp w reads pages w, w+W, ...; lane l's j-th element is word         */
+/* (page*P/E + 32j + l); a 16-B element is four independent words.       */
+/* FFT is the plain O(n^2) DFT in double (tolerance in the test).        */
+/* ------------------------------------------------------------------ */
+#include <math.h>
+#ifndef M_PI
+#define M_PI 3.14159265358979323846
+#endif
+
+static uint32_t or_lcg_n(uint32_t x, uint32_t n) {
+    for (uint32_t i = 0; i < n; ++i) x = x * 1664525u + 1013904223u;
+    return x;
+}
+
+static int or_cmp_u32(const void* a, const void* b) {
+    uint32_t x = *(const uint32_t*)a, y = *(const uint32_t*)b;
+    return x < y ? -1 : x > y;
+}
+
+/* contribution of one 32-word vector x (one word per lane) to each lane */
+static void or_work_vec(int work, const uint32_t* x, const uint32_t* x2, uint32_t iters,
+                        double* add_lane) {
+    if (work == 0) {
+        for (int l = 0; l < 32; ++l) add_lane[l] += (double)x[l] + (double)x2[l];
+    } else if (work == 1) {
+        for (int l = 0; l < 32; ++l) add_lane[l] += (double)x[l];
+    } else if (work == 2) {
+        for (int l = 0; l < 32; ++l) add_lane[l] += (double)or_lcg_n(x[l], iters);
+    } else if (work == 3) {
+        uint32_t s = 0;
+        for (int l = 0; l < 32; ++l) s += x[l];
+        for (int l = 0; l < 32; ++l) add_lane[l] += (double)s;
+    } else if (work == 4) {
+        for (int k = 0; k < 32; ++k) {
+            double re = 0, im = 0;
+            for (int n = 0; n < 32; ++n) {
+                double xr = (double)(x[n] & 0xffffu), xi = (double)(x[n] >> 16);
+                double ang = -2.0 * M_PI * (double)(n * k % 32) / 32.0;
+                re += xr * cos(ang) - xi * sin(ang);
+                im += xr * sin(ang) + xi * cos(ang);
+            }
+            add_lane[k] += floor((re * re + im * im) / 65536.0);
+        }
+    } else {
+        uint32_t s[32];
+        memcpy(s, x, sizeof s);
+        qsort(s, 32, sizeof(uint32_t), or_cmp_u32);
+        for (int l = 0; l < 32; ++l) add_lane[l] += (double)s[l] * (double)(l + 1);
+    }
+}
+
+/* acc[t] (as double; integer workloads are exact below 2^53) */
+void or_compute(const uint8_t* file, uint64_t span, uint32_t unit, uint32_t elem,
+                uint64_t nthreads, int work, uint32_t iters, double* acc, int threads) {
+    uint64_t W = nthreads / 32;
+    uint64_t nunits = span / unit;
+    uint32_t per_unit = unit / (32 * elem);
+    uint64_t second = span / 4; /* in words */
+    const uint32_t* words = (const uint32_t*)file;
+    #pragma omp parallel for schedule(dynamic, 1) num_threads(threads)
+    for (int64_t w = 0; w < (int64_t)W; ++w) {
+        double lanes[32] = {0};
+        for (uint64_t u = (uint64_t)w; u < nunits; u += W)
+            for (uint32_t j = 0; j < per_unit; ++j)
+                for (uint32_t q = 0; q < elem / 4; ++q) {
+                    uint32_t x[32], x2[32];
+                    for (int l = 0; l < 32; ++l) {
+                        uint64_t e = u * (unit / elem) + 32ull * j + l; /* element index */
+                        uint64_t wi = e * (elem / 4) + q;               /* word index */
+                        x[l] = words[wi];
+                        x2[l] = work == 0 ? words[wi + second] : 0;
+                    }
+                    or_work_vec(work, x, x2, iters, lanes);
+                }
+        for (int l = 0; l < 32; ++l) acc[w * 32 + l] = lanes[l];
+    }
+}

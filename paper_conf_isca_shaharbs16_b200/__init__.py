@@ -180,6 +180,17 @@ def ap_bench_read_host(cache, region, cfg, out_host):
     return sec.value
 
 
+WORKS = {"add": 0, "read": 1, "random": 2, "reduce": 3, "fft": 4, "bitonic": 5}
+
+
+def ap_bench_compute(cache, region, work, elem_bytes, grid, block, span_bytes, out_dev, iters=0,
+                     mode=AP_MODE_APOINTER, raw_base=None, stream=None):
+    cfg = _lib.ap_compute_cfg(WORKS.get(work, work), elem_bytes, grid, block, iters, span_bytes,
+                              mode, _ptr(raw_base))
+    _lib.check("ap_bench_compute", _lib.lib().ap_bench_compute(cache, region, ctypes.byref(cfg),
+                                                               _ptr(out_dev), _stream(stream)))
+
+
 def ap_bench_latency(cache, region, op, reps=1000):
     """Returns (cycles per op, empty timing-pair cycles)."""
     out = (ctypes.c_uint64 * 2)()

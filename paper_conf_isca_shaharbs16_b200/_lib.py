@@ -46,6 +46,11 @@ class ap_collage_in(ctypes.Structure):
                 ("raw_base", vp), ("schedule", i32)]
 
 
+class ap_compute_cfg(ctypes.Structure):
+    _fields_ = [("work", i32), ("elem_bytes", u32), ("grid", u32), ("block", u32),
+                ("iters", u32), ("span_bytes", u64), ("mode", i32), ("raw_base", vp)]
+
+
 class APError(RuntimeError):
     def __init__(self, fn, code, msg):
         super().__init__(f"{fn} failed: {code} ({msg})")
@@ -86,6 +91,7 @@ def lib():
             "ap_collage_run": (ci, [vp, u32, ctypes.POINTER(ap_collage_in), vp, vp]),
             "ap_bench_latency": (ci, [vp, u32, ci, u32, ctypes.POINTER(u64)]),
             "ap_mmap_prot": (ci, [vp, vp, u64, ci, ctypes.POINTER(u32)]),
+            "ap_bench_compute": (ci, [vp, u32, ctypes.POINTER(ap_compute_cfg), vp, vp]),
             "ap_msync": (ci, [vp, u32]),
             "ap_bench_write": (ci, [vp, u32, ctypes.POINTER(ap_bench_cfg), vp]),
             "ap_bench_copy": (ci, [vp, u32, u32, ctypes.POINTER(ap_bench_cfg), vp]),
@@ -105,7 +111,8 @@ EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", 
             "ap_cache_reset", "ap_cache_set_policy", "ap_cache_set_tuning",
             "ap_last_device_error", "ap_cache_dump", "ap_region_dump_pte", "ap_prefill",
             "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index",
-            "ap_bench_latency", "ap_mmap_prot", "ap_msync", "ap_bench_write", "ap_bench_copy"]
+            "ap_bench_latency", "ap_mmap_prot", "ap_msync", "ap_bench_write", "ap_bench_copy",
+            "ap_bench_compute"]
 
 
 def check(fn, rc):
