@@ -138,6 +138,11 @@ int ap_cache_set_policy(ap_cache_t cache, int policy, uint64_t seed);
 int ap_cache_set_tuning(ap_cache_t cache, uint32_t max_claims, uint32_t sweep_steps,
                         uint32_t timeout_ms);
 
+/* Back-off of a warp whose page is being loaded by another warp or that
+ * found no evictable frame: __nanosleep from min_ns doubling to max_ns
+ * (defaults 64 / 4096). */
+int ap_cache_set_backoff(ap_cache_t cache, uint32_t min_ns, uint32_t max_ns);
+
 /* Sticky device error word (AP_EFAULT / AP_ENOFRAME / AP_ETIMEDOUT), cleared
  * on read; AP_OK if none. Synchronises. */
 int ap_last_device_error(ap_cache_t cache);

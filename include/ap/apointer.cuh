@@ -134,6 +134,8 @@ struct alignas(64) dev_cache {
     int32_t policy;
     uint32_t max_claims;
     uint32_t sweep_steps;
+    uint32_t backoff_min_ns; /* fault-path back-off: exponential from min to max */
+    uint32_t backoff_max_ns;
 };
 
 /* ---------------------------------------------------- PTX helpers (A15) */
@@ -496,7 +498,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
     bool linked_here = false;
     bool held = !need && (x >> 63); /* linked before this call: value already loaded */
     uint64_t t0 = 0;
-    uint32_t backoff = 64;
+    uint32_t backoff = c->backoff_min_ns;
     int idle_rounds = 0;
     dev_stats* S = my_stats(c);
 
@@ -650,10 +652,10 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
                     continue;
                 }
                 __nanosleep(backoff);
-                backoff = backoff < 4096 ? backoff * 2 : 4096;
+                backoff = backoff * 2 < c->backoff_max_ns ? backoff * 2 : c->backoff_max_ns;
             } else {
                 idle_rounds = 0;
-                backoff = 64;
+                backoff = c->backoff_min_ns;
             }
         }
     }

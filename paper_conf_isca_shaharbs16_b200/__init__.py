@@ -126,6 +126,10 @@ def ap_cache_set_tuning(cache, max_claims=1, sweep_steps=64, timeout_ms=0):
                _lib.lib().ap_cache_set_tuning(cache, max_claims, sweep_steps, timeout_ms))
 
 
+def ap_cache_set_backoff(cache, min_ns=64, max_ns=4096):
+    _lib.check("ap_cache_set_backoff", _lib.lib().ap_cache_set_backoff(cache, min_ns, max_ns))
+
+
 def ap_last_device_error(cache):
     return _lib.lib().ap_last_device_error(cache)
 

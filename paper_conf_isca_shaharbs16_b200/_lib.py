@@ -81,6 +81,7 @@ def lib():
             "ap_cache_reset": (ci, [vp]),
             "ap_cache_set_policy": (ci, [vp, ci, u64]),
             "ap_cache_set_tuning": (ci, [vp, u32, u32, u32]),
+            "ap_cache_set_backoff": (ci, [vp, u32, u32]),
             "ap_last_device_error": (ci, [vp]),
             "ap_cache_dump": (ci, [vp, vp, ctypes.POINTER(u64)]),
             "ap_region_dump_pte": (ci, [vp, u32, vp]),
@@ -112,7 +113,7 @@ EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", 
             "ap_last_device_error", "ap_cache_dump", "ap_region_dump_pte", "ap_prefill",
             "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index",
             "ap_bench_latency", "ap_mmap_prot", "ap_msync", "ap_bench_write", "ap_bench_copy",
-            "ap_bench_compute"]
+            "ap_bench_compute", "ap_cache_set_backoff"]
 
 
 def check(fn, rc):

@@ -208,6 +208,8 @@ extern "C" int ap_cache_create(uint64_t frames, uint32_t page_size, int device, 
     c->h.policy = ap::POLICY_CLOCK;
     c->h.max_claims = 1;
     c->h.sweep_steps = 64;
+    c->h.backoff_min_ns = 64;
+    c->h.backoff_max_ns = 4096;
     if (push_descriptor(c) != AP_OK) return fail(AP_ECUDA);
     if (cudaDeviceSynchronize() != cudaSuccess) return fail(AP_ECUDA);
     *out = c;
@@ -426,6 +428,15 @@ extern "C" int ap_cache_set_tuning(ap_cache_t c, uint32_t max_claims, uint32_t s
     c->h.max_claims = max_claims;
     c->h.sweep_steps = sweep_steps;
     c->h.timeout_ns = (uint64_t)(timeout_ms ? timeout_ms : 20000) * 1000000ull;
+    return push_descriptor(c);
+}
+
+extern "C" int ap_cache_set_backoff(ap_cache_t c, uint32_t min_ns, uint32_t max_ns) {
+    if (!c || min_ns == 0 || max_ns < min_ns || max_ns > 1000000) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    c->h.backoff_min_ns = min_ns;
+    c->h.backoff_max_ns = max_ns;
     return push_descriptor(c);
 }
 
