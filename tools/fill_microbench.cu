@@ -30,6 +30,32 @@ __global__ void __launch_bounds__(512) k_ldg(const uint4* __restrict__ src, uint
     }
 }
 
+template <int FLAV, int U>
+__global__ void __launch_bounds__(512) k_ldg2(const uint4* __restrict__ src, uint4* __restrict__ dst,
+                                              uint64_t nchunks, uint32_t chunk) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const unsigned lane = threadIdx.x & 31;
+    const uint32_t nvec = chunk / 16;
+    for (uint64_t c = warp; c < nchunks; c += nw) {
+        const uint4* s = src + c * nvec;
+        uint4* d = dst + c * nvec;
+        for (uint32_t i = lane; i < nvec; i += 32 * U) {
+            uint4 v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const uint4* p = s + i + 32 * u;
+                if (FLAV == 0) v[u] = __ldcs(p);
+                else if (FLAV == 1) asm volatile("ld.global.nc.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v[u].x), "=r"(v[u].y), "=r"(v[u].z), "=r"(v[u].w) : "l"(p));
+                else if (FLAV == 2) asm volatile("ld.global.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v[u].x), "=r"(v[u].y), "=r"(v[u].z), "=r"(v[u].w) : "l"(p));
+                else asm volatile("ld.global.cg.L2::128B.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v[u].x), "=r"(v[u].y), "=r"(v[u].z), "=r"(v[u].w) : "l"(p));
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) __stcg(d + i + 32 * u, v[u]);
+        }
+    }
+}
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
@@ -133,6 +159,25 @@ int main(int argc, char** argv) {
             CK(cudaGetLastError());
             printf("ldg   chunk %6u grid %3d  %.2f GB/s\n", chunk, blocks, bytes / ms / 1e6);
         }
+    }
+    {
+        const uint32_t chunk = 4096;
+        const uint64_t n = bytes / chunk;
+        auto run = [&](auto kern, const char* name) {
+            for (int i = 0; i < 3; ++i) {
+                cudaEventRecord(e0);
+                kern<<<148, 512>>>((const uint4*)hd, (uint4*)d, n, chunk);
+                cudaEventRecord(e1);
+                cudaEventSynchronize(e1);
+                cudaEventElapsedTime(&ms, e0, e1);
+            }
+            printf("%-28s %.2f GB/s\n", name, bytes / ms / 1e6);
+        };
+        run(k_ldg2<0, 8>, "ld.cs unroll8");
+        run(k_ldg2<0, 4>, "ld.cs unroll4");
+        run(k_ldg2<1, 8>, "ld.nc.L2::256B unroll8");
+        run(k_ldg2<2, 8>, "ld.L2::256B unroll8");
+        run(k_ldg2<3, 8>, "ld.cg.L2::128B unroll8");
     }
     for (uint32_t chunk : {2048u, 4096u, 8192u}) {
         size_t sm = 16 * 2 * chunk;
