@@ -310,7 +310,9 @@ def emit_collage(args, res_all, world, METRIC):
         "e2e": {"value": round(max(np.mean(r["e2e"]) for r in res_all), 6), "unit": "s",
                 "h2d_bytes_per_step": r0["h2d"], "d2h_bytes_per_step": r0["d2h"],
                 "api": "target H2D + ap_collage_run + winners D2H (cold cache)"},
-        "gpu_launches": args.steps,
+        "gpu_launches": args.steps * (3 if args.schedule else 1),
+        "gpu_launches_note": "per step: k_collage (+ k_collage_keys and k_iota32 for the LSH "
+                             "schedule; the schedule's radix sort adds cub library kernels)",
         "clocks": r0["clocks"],
     }
     if r0["raw"]:

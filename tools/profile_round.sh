@@ -13,7 +13,15 @@ timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_se
   -o gpurun_out/full_hit python tools/prof_hit.py 65536 2 > gpurun_out/full_hit.out 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_seq -s 6 -c 1 \
   -o gpurun_out/full_hit_raw python tools/prof_hit.py 65536 2 > gpurun_out/full_hit_raw.out 2>&1
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_collage -s 1 -c 1 \
+timeout 900 ncu --set full --import-source on --clock-control none -k 'regex:^k_collage$' -s 1 -c 1 \
   -o gpurun_out/full_c4 python bench.py --workload c4 --steps 1 --warmup 1 --no-cpu-baseline \
   > gpurun_out/full_c4.out 2>&1
 echo done
+# bench lines (outside ncu): default C2, C1, C3, C4, C4 unaligned, C5 (1 GPU)
+timeout 600 python bench.py > gpurun_out/final_c2.json 2> gpurun_out/final_c2.err
+for w in c1 c3 c4; do timeout 900 python bench.py --workload $w > gpurun_out/final_$w.json 2> gpurun_out/final_$w.err; done
+timeout 900 python bench.py --workload c4 --stride 3072 > gpurun_out/final_c4u.json 2> gpurun_out/final_c4u.err
+timeout 1500 python bench.py --workload c5 --steps 3 --warmup 1 > gpurun_out/final_c5.json 2> gpurun_out/final_c5.err
+timeout 300 python bench.py --impl reference > gpurun_out/final_ref.json 2> gpurun_out/final_ref.err
+timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/final_smoke.txt 2>&1
+echo bench-done
