@@ -175,7 +175,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         ap.ap_prefill(big, rb, 0, npages, stream)
         torch.cuda.synchronize()
         res_g = {}
-        for g in (1, 2, 4):
+        for g in (1, 2, 4, 8):
             inp_g = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                                   cfg["N"], cfg["stride"], group=g, block_begin=b0,
                                   block_count=b1 - b0, schedule=args.schedule)

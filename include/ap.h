@@ -273,7 +273,7 @@ typedef struct {
     const uint32_t* ids_dev;     /* [L][N] record ids, ascending per bucket        */
     uint64_t N;                  /* records in the file                            */
     uint32_t rec_stride;         /* bytes between records (4096 = padded, 3072)   */
-    uint32_t group;              /* candidates per warp iteration: 1, 2 or 4       */
+    uint32_t group;              /* candidates per warp iteration: 1, 2, 4 or 8    */
     uint64_t block_begin;        /* first query block (row-major 32x32 blocks)     */
     uint64_t block_count;        /* number of query blocks                        */
     int32_t mode;                /* AP_MODE_APOINTER | AP_MODE_RAW                 */

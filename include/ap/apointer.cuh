@@ -62,6 +62,16 @@
 #endif
 #endif
 
+/* Unlink (a match, a popc and one release add per page) is inlined unless
+ * -DAP_UNLINK_NOINLINE. */
+#ifndef AP_UNLINK_ATTR
+#ifdef AP_UNLINK_NOINLINE
+#define AP_UNLINK_ATTR __noinline__
+#else
+#define AP_UNLINK_ATTR __forceinline__
+#endif
+#endif
+
 namespace ap {
 
 /* ------------------------------------------------------------ layouts */
@@ -278,7 +288,7 @@ __device__ __forceinline__ int nth_set(unsigned m, int k) {
 /* -------------------------------------------------------------------------
  * S10 unlink: lanes with `mine` drop their link to
  * `page` of `r`.  Warp-aggregated: one release-add of -n per distinct page. */
-static __device__ AP_SLOW_ATTR void unlink_lanes(unsigned m, bool mine, const dev_region* r,
+static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const dev_region* r,
                                           uint64_t page) {
     unsigned long long key = mine ? (((unsigned long long)r->id << 48) | page) : ~0ull;
     unsigned grp = __match_any_sync(m, key);
@@ -662,6 +672,63 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
     return slow_out<T>{x, page, vv};
 }
 
+/* -------------------------------------------------------------------------
+ * S5+S6 inline: the minor-fault fast path.  The unlinked lanes of m group by
+ * page (__match_any_sync), each group's leader links with one acquire add of
+ * the group size on the PTE (the same optimistic link deref_slow does, R-A17),
+ * and if the entry was VALID the lanes link to its frame.  A leader that
+ * finds the page not resident undoes its add and leaves its lanes unlinked.
+ * Returns true when every lane of m is linked afterwards; otherwise the
+ * caller runs the full fault path (deref_slow), which takes lanes linked
+ * here as already served.  Inline and call-free, so in the common resident
+ * case no register state is saved around an out-of-line call. */
+template <class T>
+__device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& page,
+                                           const dev_region* r, uint32_t lg) {
+    const bool need = !(x >> 63);
+    /* out-of-range / misaligned offsets: the full path reports them */
+    if (__any_sync(m, need && (x + sizeof(T) > r->bytes || (x % sizeof(T)) != 0))) return false;
+    const uint64_t pg = x >> lg;
+    const unsigned grp = __match_any_sync(m, need ? (((unsigned long long)r->id << 48) | pg) : ~0ull);
+    const int leader = __ffs(grp) - 1;
+    const bool is_leader = need && (int)lane_id() == leader;
+    uint64_t old = 0;
+    if (is_leader) {
+        uint64_t* pte = r->pte + pg;
+        old = add_acquire(pte, __popc(grp));
+        if ((old >> 62) == 2) {
+            if (!(old & PTE_REF)) red_or_relaxed(pte, PTE_REF);
+        } else {
+            red_add_relaxed(reinterpret_cast<unsigned long long*>(pte),
+                            (unsigned long long)(0 - (uint64_t)__popc(grp)));
+        }
+    }
+    const unsigned linkedm = __ballot_sync(m, is_leader && (old >> 62) == 2);
+    if (linkedm && (int)lane_id() == __ffs(m) - 1)
+        stat_add(&my_stats(r->cache)->minor, __popc(linkedm));
+    old = __shfl_sync(m, old, leader);
+    const bool ok = !need || (old >> 62) == 2;
+    if (need && ok) {
+        const uint64_t P = 1ull << lg;
+        const uint64_t f = (old >> 32) & PTE_FRAME_MASK;
+        x = XL_VALID | ((uint64_t)(r->pool + f * P) + (x & (P - 1)));
+        page = pg;
+    }
+    return __all_sync(m, ok);
+}
+
+/* link_minor unless built with -DAP_NO_LINK_MINOR (ablation: every link
+ * through the out-of-line fault path) */
+template <class T>
+__device__ __forceinline__ bool try_link_minor(unsigned m, uint64_t& x, uint64_t& page,
+                                               const dev_region* r, uint32_t lg) {
+#ifdef AP_NO_LINK_MINOR
+    return false;
+#else
+    return link_minor<T>(m, x, page, r, lg);
+#endif
+}
+
 template <class T, int N>
 struct tile_out {
     T v[N];
@@ -876,6 +943,8 @@ struct ptr {
         const T* a = v ? reinterpret_cast<const T*>(x & XL_ADDR) : reinterpret_cast<const T*>(r);
         T val = detail::ld_data<T>(a); /* speculative prefetch */
         if (__all_sync(m, v)) return val;
+        if (detail::try_link_minor<T>(m, x, page, r, lg))
+            return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
         const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
         x = o.x;
         page = o.page;
@@ -954,7 +1023,7 @@ struct ptr {
         const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
         bool ok = linked() && ((x ^ (x + span)) >> lg) == 0;
         if (!__all_sync(m, ok)) {
-            if (__any_sync(m, !linked())) {
+            if (__any_sync(m, !linked()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
                 const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
                 x = o.x;
                 page = o.page;
@@ -987,7 +1056,7 @@ struct ptr {
         const uint64_t last = bytes ? bytes - 1 : 0;
         bool ok = linked() && ((x ^ (x + last)) >> lg) == 0;
         if (!__all_sync(m, ok)) {
-            if (__any_sync(m, !linked())) {
+            if (__any_sync(m, !linked()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
                 const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
                 x = o.x;
                 page = o.page;

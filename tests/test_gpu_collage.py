@@ -48,7 +48,7 @@ def test_index_matches_oracle(ap, K, bb):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1)])
+@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1)])
 @pytest.mark.parametrize("frames", [48, 5000])
 def test_collage_matches_oracle(ap, group, schedule, frames):
     dev = torch.device("cuda:0")
@@ -116,7 +116,7 @@ def test_collage_partitioned_blocks_equal_whole(ap):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group", [1, 2, 4])
+@pytest.mark.parametrize("group", [1, 2, 4, 8])
 @pytest.mark.parametrize("frames", [40, 3000])
 def test_unaligned_records_collage(ap, group, frames):
     """NEXT N1: 3 KiB histograms without padding, so records

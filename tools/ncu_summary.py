@@ -38,7 +38,7 @@ for rr in raw[2:]:
 src = list(csv.reader(io.StringIO(ncu("--page", "source", "--csv", "--print-source", "sass"))))
 h = src[1]
 i_src, i_s, i_e = h.index("Source"), h.index("Warp Stall Sampling (All Samples)"), h.index("Instructions Executed")
-data = [r for r in src[2:] if len(r) == len(h)]
+data = [r for r in src[2:] if len(r) == len(h) and r[i_s].isdigit()]
 tot = sum(int(r[i_s]) for r in data) or 1
 print(f"top stall PCs (of {tot} samples):")
 for r in sorted(data, key=lambda r: -int(r[i_s]))[:topn]:
