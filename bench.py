@@ -259,15 +259,56 @@ def run_hit(args, torch, dev, ap, cache, region, f, stream, span=GiB, passes=8):
     res = dict(bytes_per_launch=nbytes, raw_s=float(np.mean(t_raw)),
                raw_gbs=nbytes / np.mean(t_raw) / 1e9)
     same = True
-    for acc, name in ((ap.AP_ACCESS_TILE, "tile"), (ap.AP_ACCESS_RANGE, "range"),
-                      (ap.AP_ACCESS_DEREF, "deref")):
+    for acc, name in ((ap.AP_ACCESS_TILE, "tile"), (ap.AP_ACCESS_RANGE, "range")):
         cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=page, passes=passes,
                            span_bytes=span, access=acc)
         t = run(cfg, out)
         same = same and bool(torch.equal(out, out_raw))
         res[name] = dict(s=float(np.mean(t)), gbs=nbytes / np.mean(t) / 1e9,
                          overhead=float(np.mean(t) / np.mean(t_raw) - 1))
+    # per-access form: one load in flight per warp, so it runs at full
+    # occupancy (4 CTAs of 512 per SM); its twin is the same per-access loop
+    # on a raw pointer at the same launch
+    grid_d = 4 * 148
+    out_d = torch.empty(grid_d * block, dtype=torch.int64, device=dev)
+    out_rd = torch.empty_like(out_d)
+    cfg_rd = ap.bench_cfg(ap.AP_SEQ, 16, grid_d, block, unit_bytes=page, passes=passes,
+                          span_bytes=span, mode=ap.AP_MODE_RAW, raw_base=dcopy.data_ptr(),
+                          access=ap.AP_ACCESS_DEREF)
+    cfg_d = ap.bench_cfg(ap.AP_SEQ, 16, grid_d, block, unit_bytes=page, passes=passes,
+                         span_bytes=span, access=ap.AP_ACCESS_DEREF)
+    t_rd = run(cfg_rd, out_rd)
+    t = run(cfg_d, out_d)
+    same = same and bool(torch.equal(out_d, out_rd))
+    res["deref"] = dict(s=float(np.mean(t)), gbs=nbytes / np.mean(t) / 1e9,
+                        overhead=float(np.mean(t) / np.mean(t_raw) - 1),
+                        raw_deref_gbs=nbytes / np.mean(t_rd) / 1e9,
+                        overhead_vs_raw_deref=float(np.mean(t) / np.mean(t_rd) - 1), grid=grid_d)
     st1 = ap.ap_cache_stats(cache)
+    # M2r: uniform-random 4-B reads over the resident GiB, so
+    # every read leaves its page: an unlink + a minor fault per read, vs the
+    # raw gather from the HBM copy.  Full occupancy for both (one read in
+    # flight per thread between faults).
+    grid_m, reads_m = 4 * 148, 8
+    out_m = torch.empty(grid_m * block, dtype=torch.int64, device=dev)
+    out_mr = torch.empty_like(out_m)
+    cfg_m = ap.bench_cfg(ap.AP_UNIFORM, 4, grid_m, block, reads_per_thread=reads_m, seed=11,
+                         span_bytes=span)
+    cfg_mr = ap.bench_cfg(ap.AP_UNIFORM, 4, grid_m, block, reads_per_thread=reads_m, seed=11,
+                          span_bytes=span, mode=ap.AP_MODE_RAW, raw_base=dcopy.data_ptr())
+    st_m0 = ap.ap_cache_stats(cache)
+    t_m = run(cfg_m, out_m)
+    st_m1 = ap.ap_cache_stats(cache)
+    t_mr = run(cfg_mr, out_mr)
+    nreads = grid_m * block * reads_m
+    res["minor"] = dict(
+        reads_per_launch=nreads, s=float(np.mean(t_m)), raw_s=float(np.mean(t_mr)),
+        reads_per_s=nreads / np.mean(t_m), raw_reads_per_s=nreads / np.mean(t_mr),
+        useful_gbs=4 * nreads / np.mean(t_m) / 1e9, sector_gbs=32 * nreads / np.mean(t_m) / 1e9,
+        overhead=float(np.mean(t_m) / np.mean(t_mr) - 1),
+        majors=st_m1["major"] - st_m0["major"],
+        minors_per_launch=(st_m1["minor"] - st_m0["minor"]) / max(1, len(t_m) + max(args.warmup, 3)),
+        equal_raw=bool(torch.equal(out_m, out_mr)), grid=grid_m)
     del dcopy
     res.update(majors_during=st1["major"] - st0["major"], checksums_equal_raw=same,
                ap_gbs=res["tile"]["gbs"], overhead=res["tile"]["overhead"])
@@ -352,11 +393,32 @@ def emit_c2(args, res_all, rank, world):
             "access_styles": {k: {"GBps": round(hit[k]["gbs"], 1),
                                   "overhead_vs_raw": round(hit[k]["overhead"], 4)}
                               for k in ("tile", "range", "deref")},
+            "deref_vs_raw_per_access_twin": {
+                "raw_GBps": round(hit["deref"]["raw_deref_gbs"], 1),
+                "overhead": round(hit["deref"]["overhead_vs_raw_deref"], 4),
+                "grid": hit["deref"]["grid"]},
             "access_note": "tile = read_tile<16> (one translation check per 16 accesses, the "
                            "headline); range = pin_range (one check per page); deref = `v = *q; "
-                           "q += 32` one access at a time (the paper's loop, 1 load in flight)",
+                           "q += 32` one access at a time (the paper's loop, 1 load in flight "
+                           "per warp, so run at full occupancy: 4x148 CTAs of 512, 32 registers); "
+                           "overhead_vs_raw is against the tiled raw twin, "
+                           "deref_vs_raw_per_access_twin against the same per-access loop on a "
+                           "raw pointer at the same launch",
             "major_faults_during": hit["majors_during"],
             "checksums_equal_raw": hit["checksums_equal_raw"]},
+        "minor": {
+            "workload": "M2r: the same resident GiB, uniform-random 4-B apointer reads (8 per "
+                        "thread, 4x148 CTAs of 512): every read leaves its page, i.e. one unlink "
+                        "+ one minor fault (PTE atomic) per read; raw twin = the same gather "
+                        "from an HBM copy",
+            "reads_per_s": round(hit["minor"]["reads_per_s"], 1),
+            "raw_reads_per_s": round(hit["minor"]["raw_reads_per_s"], 1),
+            "useful_GBps": round(hit["minor"]["useful_gbs"], 3),
+            "sector_GBps": round(hit["minor"]["sector_gbs"], 3),
+            "overhead_vs_raw": round(hit["minor"]["overhead"], 4),
+            "major_faults_during": hit["minor"]["majors"],
+            "minor_faults_per_launch": hit["minor"]["minors_per_launch"],
+            "checksums_equal_raw": hit["minor"]["equal_raw"]},
         "roofline": {"bound": "host_link", "achieved": round(achieved, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
                      "frac": round(achieved / r0["link"], 4),

@@ -181,7 +181,7 @@ typedef struct {
     uint32_t unit_bytes;       /* SEQ: bytes per warp unit (multiple of 32*elem, *
                                 *      divides the page size)                    */
     uint32_t page_bytes;       /* DIVERGENT: page size of the pattern            */
-    uint64_t span_bytes;       /* SEQ: bytes swept (0 = whole region)            */
+    uint64_t span_bytes;       /* SEQ: bytes swept; UNIFORM: offsets drawn from [0, span_bytes); 0 = whole region */
     uint64_t seed;             /* UNIFORM / DIVERGENT offset generator seed       */
     int32_t mode;              /* AP_MODE_APOINTER | AP_MODE_RAW                 */
     int32_t out_copy;          /* SEQ: out receives the bytes read at their      *

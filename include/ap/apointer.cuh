@@ -72,6 +72,16 @@
 #endif
 #endif
 
+/* Speculative load of the hit path; -DAP_SPECULATIVE=0 is
+ * the ablation that loads only after the warp's vote. */
+#ifndef AP_SPECULATIVE
+#define AP_SPECULATIVE 1
+#endif
+/* Stride prefetch distance of the per-access dereference (0 = off). */
+#ifndef AP_PREFETCH_DIST
+#define AP_PREFETCH_DIST 0
+#endif
+
 namespace ap {
 
 /* ------------------------------------------------------------ layouts */
@@ -195,6 +205,9 @@ __device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
 }
 __device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 __device__ __forceinline__ void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 __device__ __forceinline__ uint64_t cas_acquire(uint64_t* p, uint64_t cmp, uint64_t val) {
@@ -899,6 +912,7 @@ struct ptr {
     const dev_region* r; /* metadata: region                                */
     uint64_t page;       /* metadata: linked page                           */
     uint32_t lg;         /* metadata: log2(page size)                       */
+    int64_t step = 0;    /* bytes of the last += (stride predictor)         */
 
     __device__ __forceinline__ ptr() : x(0), r(nullptr), page(0), lg(12) {}
     __device__ __forceinline__ ptr(const dev_region* reg, uint32_t log2_page, uint64_t foff)
@@ -940,8 +954,23 @@ struct ptr {
     __device__ __forceinline__ T operator*() {
         const unsigned m = __activemask();
         const bool v = linked();
+#if AP_SPECULATIVE
         const T* a = v ? reinterpret_cast<const T*>(x & XL_ADDR) : reinterpret_cast<const T*>(r);
         T val = detail::ld_data<T>(a); /* speculative prefetch */
+#else
+        /* ablation: the load waits for the vote */
+        if (__all_sync(m, v)) return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
+        T val{};
+#endif
+#if AP_PREFETCH_DIST > 0
+        {
+            /* stride prefetch: the datum AP_PREFETCH_DIST steps ahead, if it
+             * is in the linked page, is requested into L2 (no register
+             * result, so nothing waits on it) */
+            const uint64_t px = x + (uint64_t)(step * AP_PREFETCH_DIST);
+            if (v && ((x ^ px) >> lg) == 0) detail::prefetch_l2(reinterpret_cast<const void*>(px & XL_ADDR));
+        }
+#endif
         if (__all_sync(m, v)) return val;
         if (detail::try_link_minor<T>(m, x, page, r, lg))
             return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
@@ -1071,6 +1100,7 @@ struct ptr {
      * unlinks with a warp-aggregated decrement (S10). */
     __device__ __forceinline__ ptr& operator+=(int64_t d) {
         const uint64_t nb = (uint64_t)(d * (int64_t)sizeof(T));
+        step = (int64_t)nb;
         const uint64_t nx = x + nb;
         const bool cross = linked() && ((x ^ nx) >> lg) != 0;
         const unsigned m = __activemask();

@@ -27,6 +27,9 @@
 #ifndef AP_BENCH_MINB
 #define AP_BENCH_MINB 1
 #endif
+#ifndef AP_SEQ_MINB
+#define AP_SEQ_MINB AP_BENCH_MINB
+#endif
 
 namespace {
 
@@ -60,7 +63,7 @@ struct BenchArgs {
 
 __device__ __forceinline__ uint64_t uniform_off(const BenchArgs& a, uint32_t E, uint64_t t,
                                                 uint64_t i) {
-    return (ap::detail::sm64(a.seed ^ (t << 24) ^ i) % (a.bytes / E)) * E;
+    return (ap::detail::sm64(a.seed ^ (t << 24) ^ i) % (a.span / E)) * E;
 }
 
 __device__ __forceinline__ uint64_t divergent_off(const BenchArgs& a, uint32_t E, uint64_t t,
@@ -148,8 +151,45 @@ __device__ __forceinline__ void seq_unit_deref(ap::ptr<T>& q, const BenchArgs& a
     }
 }
 
+/* The per-access form keeps one load in flight per warp (each access may
+ * enter the fault path), so it needs warps, not registers: this kernel is
+ * built for AP_DEREF_MINB CTAs of 512 threads per SM (full occupancy at 4,
+ * 32 registers; the out-of-line fault path spills, the hit path does not).
+ * The raw twin runs the same per-access loop on a plain pointer. */
+#ifndef AP_DEREF_MINB
+#define AP_DEREF_MINB 4
+#endif
 template <class T, bool APTR>
-__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_DEREF_MINB)
+    k_seq_deref(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t w = t >> 5, lane = t & 31;
+    const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
+    const uint32_t per_unit = a.unit / (32 * E);
+    uint64_t h = FNV_BASIS;
+    for (uint32_t pass = 0; pass < a.passes; ++pass) {
+        for (uint64_t u = w; u < nunits; u += W) {
+            const uint64_t e0 = u * (a.unit / E) + lane;
+            if constexpr (APTR) {
+                ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
+                seq_unit_deref<T>(q, a, e0, per_unit, h);
+            } else {
+                raw_reader<T> q{reinterpret_cast<const T*>(a.raw) + e0};
+                for (uint32_t j = 0; j < per_unit; ++j) {
+                    const uint64_t off = (e0 + 32ull * j) * E;
+                    if (off + E <= a.span) consume(a, off, *q, h);
+                    q += 32;
+                }
+            }
+        }
+    }
+    if (!a.out_copy) a.ck[t] = h;
+}
+
+template <class T, bool APTR>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     k_seq(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
     constexpr uint32_t E = sizeof(T);
     const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -165,9 +205,7 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
             const bool whole = (u + 1) * a.unit <= a.span;
             if constexpr (APTR) {
                 ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
-                if (a.access == AP_ACCESS_DEREF) {
-                    seq_unit_deref<T>(q, a, e0, per_unit, h);
-                } else if (a.access == AP_ACCESS_RANGE && whole) {
+                if (a.access == AP_ACCESS_RANGE && whole) {
                     /* translate once for the unit, then stream plain loads
                      * through the linked translation (valid while q lives) */
                     const T* p = q.pin_range(32ull * E * (per_unit - 1) + E);
@@ -222,7 +260,12 @@ template <class T, bool APTR>
 cudaError_t launch_t(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg,
                      const BenchArgs& a, cudaStream_t s) {
     switch (cfg->pattern) {
-        case AP_SEQ: k_seq<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a); break;
+        case AP_SEQ:
+            if (cfg->access == AP_ACCESS_DEREF)
+                k_seq_deref<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            else
+                k_seq<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            break;
         case AP_UNIFORM:
             k_random<T, AP_UNIFORM, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             break;
@@ -271,8 +314,8 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
             if (cfg->out_copy) a->out_copy = (uint8_t*)out;
             else a->ck = (uint64_t*)out;
             break;
-        case AP_UNIFORM:
-            if (rg.bytes < E) return AP_EINVAL;
+        case AP_UNIFORM: /* offsets uniform over [0, span) (span 0 = the region) */
+            if (a->span < E || a->span > rg.bytes) return AP_EINVAL;
             a->ck = (uint64_t*)out;
             break;
         case AP_DIVERGENT:

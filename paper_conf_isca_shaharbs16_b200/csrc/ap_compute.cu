@@ -120,8 +120,14 @@ __device__ __forceinline__ unsigned long long work_elem(const uint4& v, const ui
            work_word<WORK>(v.z, v2.z, lane, iters) + work_word<WORK>(v.w, v2.w, lane, iters);
 }
 
+/* per-access loops need warps, not registers: built for full occupancy
+ * (4 CTAs of 512 threads per SM, 32 registers), the sweep's upper end as in
+ * the paper's Fig. 6 x axis */
+#ifndef AP_COMPUTE_MINB
+#define AP_COMPUTE_MINB 1
+#endif
 template <class T, int WORK, bool APTR>
-__global__ void __launch_bounds__(AP_BENCH_THREADS, 1)
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_COMPUTE_MINB)
     k_compute(const ap::dev_cache* __restrict__ c, uint32_t region, const CompArgs a) {
     constexpr uint32_t E = sizeof(T);
     const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;

@@ -192,3 +192,58 @@ def test_reset_starts_cold(ap, dev):
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("elem", [4, 16])
+def test_uniform_over_resident_span_minor_faults(ap, dev, elem):
+    """M2r: offsets uniform over a resident span (span_bytes < region), every
+    read a minor fault through the inline link path; values == oracle over
+    the span, no major faults, one link per (warp, distinct page) group."""
+    page, nbytes, span = 65536, 32 << 20, 8 << 20
+    f = make_file(nbytes, seed=12)
+    cache = ap.ap_cache_create(span // page + 8, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        ap.ap_prefill(cache, r, 0, span // page)
+        torch.cuda.synchronize()
+        st0 = ap.ap_cache_stats(cache)
+        grid, block, reads = 296, 512, 5
+        cfg = ap.bench_cfg(ap.AP_UNIFORM, elem, grid, block, reads_per_thread=reads, seed=21,
+                           span_bytes=span)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_uniform(f[:span], span, elem, grid * block, reads, 21)
+        assert np.array_equal(got, want)
+        st1 = ap.ap_cache_stats(cache)
+        assert st1["major"] == st0["major"]
+        assert st1["minor"] > st0["minor"]
+        assert check_invariants(ap, cache, [r], span // page + 8) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("frames", [3, 512])
+def test_per_access_deref_kernel(ap, dev, frames):
+    """The per-access `v = *q; q += 32` kernel (full-occupancy build) and its
+    raw per-access twin both equal the oracle, with the cache smaller and
+    larger than the span."""
+    page, nbytes = 4096, 1 << 20
+    f = make_file(nbytes, seed=13)
+    cache = ap.ap_cache_create(frames, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        grid, block = 16, 512
+        cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=4096, passes=2,
+                           access=ap.AP_ACCESS_DEREF)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_seq(f, nbytes, 4096, 16, grid * block, 2)
+        assert np.array_equal(got, want)
+        dcopy = torch.from_numpy(f).to(dev)
+        cfg_raw = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=4096, passes=2,
+                               access=ap.AP_ACCESS_DEREF, mode=ap.AP_MODE_RAW,
+                               raw_base=dcopy.data_ptr())
+        assert np.array_equal(_run(ap, cache, r, cfg_raw, grid * block, dev).view(np.uint64), want)
+        assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)

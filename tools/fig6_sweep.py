@@ -11,7 +11,7 @@ import paper_conf_isca_shaharbs16_b200 as ap  # noqa: E402
 import synth  # noqa: E402
 
 page = 65536
-span = 128 << 20
+span = 1 << 30
 raw = np.empty(2 * span + (1 << 21), np.uint8)
 o = (-raw.ctypes.data) % (1 << 21)
 f = synth.fill_file(raw[o:o + 2 * span], 1)
@@ -38,7 +38,9 @@ def timed(fn, n=3):
 
 works = [("add", 0), ("read", 0), ("random", 10), ("random", 50), ("reduce", 0), ("fft", 0),
          ("bitonic", 0)]
-tbs = [1, 4, 16, 37, 74, 148]
+import os
+MINB = int(os.environ.get("AP_FIG6_MINB", 1))  # CTAs of 512 per SM the library's k_compute is built for
+tbs = [t for t in (1, 4, 16, 37, 74, 148, 296, 444, 592) if t <= 148 * MINB]
 print("# apointer overhead vs raw twin (time_ap / time_raw - 1), 512-thread blocks, "
       f"{span >> 20} MiB per vector resident, one access at a time (no tiling)")
 for elem in (4, 16):
