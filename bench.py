@@ -491,7 +491,7 @@ def main():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--group", type=int, default=8, help="collage candidates per warp (1, 2, 4, 8)")
-    p.add_argument("--schedule", type=int, default=1, help="collage: 1 = LSH-sorted blocks, 0 = natural")
+    p.add_argument("--schedule", type=int, default=2, help="collage: 0 = natural, 1 = LSH-sorted blocks, 2 = per-table units")
     p.add_argument("--stride", type=int, default=4096, help="collage record stride (3072 = unaligned)")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
     p.add_argument("--no-cpu-baseline", action="store_true")

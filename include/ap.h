@@ -282,12 +282,18 @@ typedef struct {
                                   * single kernel); AP_SCHED_LSH: blocks are first *
                                   * sorted by their LSH keys (an extra key kernel  *
                                   * + radix sort) so blocks sharing buckets run    *
-                                  * together and reuse cached records.  Results   *
-                                  * are identical (per-block argmin).             */
+                                  * together and reuse cached records;           *
+                                  * AP_SCHED_TABLE: the work unit is one block's  *
+                                  * candidates from one table, units sorted by    *
+                                  * (table, bucket), so every unit reading a      *
+                                  * bucket runs together; the block's winner is   *
+                                  * the atomic 64-bit min over its L units.       *
+                                  * Results are identical (per-block argmin).     */
 } ap_collage_in;
 
 #define AP_SCHED_NATURAL 0
 #define AP_SCHED_LSH 1
+#define AP_SCHED_TABLE 2
 
 /* ap_collage_run — the collage kernel ("calculates the
  * histogram of each 32x32 block, computes its LSH keys, reads the candidate

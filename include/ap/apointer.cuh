@@ -77,6 +77,12 @@
 #ifndef AP_SPECULATIVE
 #define AP_SPECULATIVE 1
 #endif
+/* Reference bit of a freshly filled page (second-chance clock, R-A11):
+ * 1 = set at the fill, 0 = set only when the page is linked again (a minor
+ * fault), so pages touched once are evicted before re-referenced ones. */
+#ifndef AP_REF_ON_FILL
+#define AP_REF_ON_FILL 1
+#endif
 /* Stride prefetch distance of the per-access dereference (0 = off). */
 #ifndef AP_PREFETCH_DIST
 #define AP_PREFETCH_DIST 0
@@ -611,7 +617,8 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             if ((int)lane == L) printf("[publish] w%u m%08x n%u f%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, n, f, (unsigned long long)fpg);
 #endif
             if ((int)lane == L)
-                red_add_release(pte, (PTE_VALID - PTE_LOADING) | PTE_REF | ((uint64_t)f << 32) |
+                red_add_release(pte, (PTE_VALID - PTE_LOADING) | (AP_REF_ON_FILL ? PTE_REF : 0) |
+                                         ((uint64_t)f << 32) |
                                          (uint64_t)n);
         }
         const unsigned nminor = __popc(__ballot_sync(m, st == ST_LINKED));

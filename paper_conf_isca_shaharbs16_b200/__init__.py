@@ -204,7 +204,7 @@ def ap_bench_latency(cache, region, op, reps=1000):
 
 def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev, ids_dev, N,
                rec_stride=4096, group=1, block_begin=0, block_count=None,
-               mode=AP_MODE_APOINTER, raw_base=None, L=None, K=None, schedule=1):
+               mode=AP_MODE_APOINTER, raw_base=None, L=None, K=None, schedule=AP_SCHED_TABLE):
     L = proj_dev.shape[0] if L is None else L
     K = proj_dev.shape[1] if K is None else K
     nb = (W // 32) * (H // 32)

@@ -48,7 +48,7 @@ def test_index_matches_oracle(ap, K, bb):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1)])
+@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1), (1, 2), (8, 2)])
 @pytest.mark.parametrize("frames", [48, 5000])
 def test_collage_matches_oracle(ap, group, schedule, frames):
     dev = torch.device("cuda:0")
@@ -108,7 +108,7 @@ def test_collage_partitioned_blocks_equal_whole(ap):
             part = torch.zeros((b1 - b0, 2), dtype=torch.int32, device=dev)
             ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
                                                       block_begin=b0, block_count=b1 - b0,
-                                                      schedule=g % 2), part)
+                                                      schedule=g % 3), part)
             parts.append(part)
         assert torch.equal(torch.cat(parts), full)
         ap.ap_munmap(cache, r)
@@ -116,9 +116,9 @@ def test_collage_partitioned_blocks_equal_whole(ap):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group", [1, 2, 4, 8])
+@pytest.mark.parametrize("group,schedule", [(1, 1), (2, 1), (4, 1), (8, 1), (4, 2), (8, 2)])
 @pytest.mark.parametrize("frames", [40, 3000])
-def test_unaligned_records_collage(ap, group, frames):
+def test_unaligned_records_collage(ap, group, schedule, frames):
     """NEXT N1: 3 KiB histograms without padding, so records
     straddle 4 KiB pages; the same kernel and pointers must still match the
     oracle bit for bit."""
@@ -137,7 +137,7 @@ def test_unaligned_records_collage(ap, group, frames):
         nb = (W // 32) * (H // 32)
         win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
         ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride,
-                                                  group=group), win)
+                                                  group=group, schedule=schedule), win)
         torch.cuda.synchronize()
         assert ap.ap_last_device_error(cache) == 0
         want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
