@@ -25,6 +25,9 @@ LSH_SEED, DS_SEED, TGT_SEED = 22, 21, 23
 
 def collage_config(name, stride=4096):
     cfg = _collage_config(name)
+    if os.environ.get("AP_COLLAGE_FRAMES"):  # experiments only (e.g. a cache >= the file)
+        cfg["frames"] = int(os.environ["AP_COLLAGE_FRAMES"])
+        cfg["workload"] += f"; CACHE OVERRIDE {cfg['frames']} frames"
     if stride != 4096:  # NEXT N1: unaligned 3 KiB records, no padding
         cfg["stride"] = stride
         cfg["workload"] += f"; UNALIGNED {stride}-B records (no padding, records straddle pages)"
