@@ -16,6 +16,10 @@ timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_se
 timeout 900 ncu --set full --import-source on --clock-control none -k 'regex:^k_collage$' -s 1 -c 1 \
   -o gpurun_out/full_c4 python bench.py --workload c4 --steps 1 --warmup 1 --no-cpu-baseline \
   > gpurun_out/full_c4.out 2>&1
+AP_PROF_STEPS=1 timeout 900 ncu --set full --import-source on --clock-control none -k 'regex:^k_collage$' -c 2 \
+  -o gpurun_out/full_c4_resident python tools/prof_collage.py 1048576 8 > gpurun_out/full_c4_resident.out 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_random -c 2 \
+  -o gpurun_out/full_minor python tools/prof_minor.py > gpurun_out/full_minor.out 2>&1
 echo done
 # bench lines (outside ncu): default C2, C1, C3, C4, C4 unaligned, C5 (1 GPU)
 timeout 600 python bench.py > gpurun_out/final_c2.json 2> gpurun_out/final_c2.err
@@ -24,4 +28,6 @@ timeout 900 python bench.py --workload c4 --stride 3072 > gpurun_out/final_c4u.j
 timeout 1500 python bench.py --workload c5 --steps 3 --warmup 1 > gpurun_out/final_c5.json 2> gpurun_out/final_c5.err
 timeout 300 python bench.py --impl reference > gpurun_out/final_ref.json 2> gpurun_out/final_ref.err
 timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/final_smoke.txt 2>&1
+timeout 600 python tools/fig6_sweep.py > gpurun_out/final_fig6.txt 2>&1
+timeout 300 python tools/latency.py > gpurun_out/final_latency.txt 2>&1
 echo bench-done
