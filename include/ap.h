@@ -224,7 +224,10 @@ int ap_bench_write(ap_cache_t cache, ap_region_t region, const ap_bench_cfg* cfg
 
 /* ap_bench_copy — dst[e] = src[e] for the SEQ pattern of cfg, reading and
  * writing through apointers (the copy kernel of PAPER.md:310-316).  dst must
- * be writable.  Asynchronous on `stream`. */
+ * be writable.  cfg->mode = AP_MODE_RAW runs the raw twin (the same loop on
+ * plain pointers): cfg->raw_base is a device buffer of 2 * span bytes, src =
+ * its first half, dst = its second half (the regions are only validated).
+ * Asynchronous on `stream`. */
 int ap_bench_copy(ap_cache_t cache, ap_region_t src, ap_region_t dst, const ap_bench_cfg* cfg,
                   void* stream);
 

@@ -1015,12 +1015,22 @@ struct ptr {
             for (int k = 0; k < N; ++k) detail::st_data<T>(a + k * stride, v[k]);
             return;
         }
+        /* slow path: the values go to a local array first, so no register
+         * holding them is live across a call (ptxas would otherwise spill the
+         * tile right after its loads, on the fast path too) */
+        T tmp[N];
+#pragma unroll
+        for (int k = 0; k < N; ++k) tmp[k] = v[k];
+        write_tile_slow<N>(*this, tmp, stride);
+    }
+    template <int N>
+    static __device__ __noinline__ void write_tile_slow(ptr& p, const T* v, int64_t stride) {
 #pragma unroll 1
         for (int k = 0; k < N; ++k) {
-            store(v[k]);
-            *this += stride;
+            p.store(v[k]);
+            p += stride;
         }
-        *this -= N * stride;
+        p -= N * stride;
     }
 
     /* warp-wide: every active lane is linked (and, for stores, marked dirty) */

@@ -568,7 +568,7 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
 
 /* dst[e] = src[e] for e < span/E, both through apointers (the copy kernel
  * of PAPER.md:312: tiled reads, stores one element at a time). */
-template <class T>
+template <class T, bool APTR>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
     k_copy(const ap::dev_cache* __restrict__ c, uint32_t src, uint32_t dst, const BenchArgs a) {
     constexpr uint32_t E = sizeof(T);
@@ -578,34 +578,56 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
     const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
     const uint32_t per_unit = a.unit / (32 * E);
-    for (uint64_t u = w; u < nunits; u += W) {
-        const uint64_t e0 = u * (a.unit / E) + lane;
-        const bool whole = (u + 1) * a.unit <= a.span;
-        ap::ptr<T> s = ap::gvmmap<T>(c, src, e0 * E);
-        ap::ptr<T> d = ap::gvmmap<T>(c, dst, e0 * E);
-        uint32_t j = 0;
-        if (whole) {
-            for (; j + CT <= per_unit; j += CT) {
-                T v[CT];
-                /* never hold one pin while the other pointer faults on a
-                 * recycled cache (R-A19): drop it first under pressure */
-                if (!s.linked_all() && d.cache_pressure()) d.release();
-                s.read_tile(v, 32);
-                if (!d.store_ready() && s.cache_pressure()) s.release();
-                d.write_tile(v, 32);
-                s += 32 * CT;
-                d += 32 * CT;
+    if constexpr (!APTR) {
+        /* raw twin: the same loop on plain pointers (src = raw, dst = raw + span) */
+        const T* sp = reinterpret_cast<const T*>(a.raw);
+        T* dp = reinterpret_cast<T*>(const_cast<uint8_t*>(a.raw) + a.span);
+        for (uint64_t u = w; u < nunits; u += W) {
+            const uint64_t e0 = u * (a.unit / E) + lane;
+            uint32_t j = 0;
+            if ((u + 1) * a.unit <= a.span) {
+                for (; j + CT <= per_unit; j += CT) {
+                    T v[CT];
+#pragma unroll
+                    for (int k = 0; k < CT; ++k) v[k] = ap::detail::ld_data<T>(sp + e0 + 32ull * (j + k));
+#pragma unroll
+                    for (int k = 0; k < CT; ++k) ap::detail::st_data<T>(dp + e0 + 32ull * (j + k), v[k]);
+                }
             }
+            for (; j < per_unit; ++j)
+                if ((e0 + 32ull * j + 1) * E <= a.span)
+                    ap::detail::st_data<T>(dp + e0 + 32ull * j, ap::detail::ld_data<T>(sp + e0 + 32ull * j));
         }
-        for (; j < per_unit; ++j) {
-            if ((e0 + 32ull * j + 1) * E <= a.span) {
-                const T v = *s;
-                if (s.cache_pressure()) s.release();
-                d.store(v);
-                if (d.cache_pressure()) d.release();
+    } else {
+        for (uint64_t u = w; u < nunits; u += W) {
+            const uint64_t e0 = u * (a.unit / E) + lane;
+            const bool whole = (u + 1) * a.unit <= a.span;
+            ap::ptr<T> s = ap::gvmmap<T>(c, src, e0 * E);
+            ap::ptr<T> d = ap::gvmmap<T>(c, dst, e0 * E);
+            uint32_t j = 0;
+            if (whole) {
+                for (; j + CT <= per_unit; j += CT) {
+                    T v[CT];
+                    /* never hold one pin while the other pointer faults on a
+                     * recycled cache (R-A19): drop it first under pressure */
+                    if (!s.linked_all() && d.cache_pressure()) d.release();
+                    s.read_tile(v, 32);
+                    if (!d.store_ready() && s.cache_pressure()) s.release();
+                    d.write_tile(v, 32);
+                    s += 32 * CT;
+                    d += 32 * CT;
+                }
             }
-            s += 32;
-            d += 32;
+            for (; j < per_unit; ++j) {
+                if ((e0 + 32ull * j + 1) * E <= a.span) {
+                    const T v = *s;
+                    if (s.cache_pressure()) s.release();
+                    d.store(v);
+                    if (d.cache_pressure()) d.release();
+                }
+                s += 32;
+                d += 32;
+            }
         }
     }
 }
@@ -671,14 +693,27 @@ extern "C" int ap_bench_copy(ap_cache_t c, ap_region_t src, ap_region_t dst,
     if (a.unit == 0 || a.unit % (32 * E) || c->page % a.unit || a.span > a.bytes ||
         a.span > c->reg[dst].bytes)
         return AP_EINVAL;
+    if (cfg->mode == AP_MODE_RAW) {
+        if (!cfg->raw_base) return AP_EINVAL;
+        a.raw = (const uint8_t*)cfg->raw_base; /* src; dst = raw_base + span */
+    } else if (cfg->mode != AP_MODE_APOINTER) {
+        return AP_EINVAL;
+    }
     ap_device_guard g(c->device);
     cudaStream_t s = (cudaStream_t)stream;
+    const bool aptr = cfg->mode == AP_MODE_APOINTER;
     switch (E) {
-        case 4: k_copy<uint32_t><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a); break;
-        case 8:
-            k_copy<unsigned long long><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+        case 4:
+            if (aptr) k_copy<uint32_t, true><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+            else k_copy<uint32_t, false><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
             break;
-        default: k_copy<uint4><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+        case 8:
+            if (aptr) k_copy<unsigned long long, true><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+            else k_copy<unsigned long long, false><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+            break;
+        default:
+            if (aptr) k_copy<uint4, true><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
+            else k_copy<uint4, false><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, src, dst, a);
     }
     AP_CUDA_TRY(cudaGetLastError());
     return AP_OK;

@@ -45,11 +45,20 @@ b = torch.empty_like(a)
 tm = t(lambda: b.copy_(a))
 print(f"# B200 copy bandwidth (read+write bytes / time), {span >> 20} MiB, pages resident")
 print(f"cudaMemcpy D2D (torch copy_): {2 * span / tm / 1e9:.1f} GB/s")
+both = torch.empty(2 * span, dtype=torch.uint8, device="cuda")
+both[:span].copy_(torch.from_numpy(src))
+import os  # noqa: E402
+grid = int(os.environ.get("AP_GRID", 148))
 for elem in (4, 8, 16):
-    cfg = ap.bench_cfg(ap.AP_SEQ, elem, 148, 512, unit_bytes=page, span_bytes=span)
+    cfg = ap.bench_cfg(ap.AP_SEQ, elem, grid, 512, unit_bytes=page, span_bytes=span)
+    cfg_r = ap.bench_cfg(ap.AP_SEQ, elem, grid, 512, unit_bytes=page, span_bytes=span,
+                         mode=ap.AP_MODE_RAW, raw_base=both.data_ptr())
     ta = t(lambda: ap.ap_bench_copy(c, rs, rd, cfg))
+    tr = t(lambda: ap.ap_bench_copy(c, rs, rd, cfg_r))
     print(f"apointer copy {elem:2d}-B: {2 * span / ta / 1e9:.1f} GB/s "
-          f"({tm / ta * 100:.1f}% of cudaMemcpy)")
+          f"({tm / ta * 100:.1f}% of cudaMemcpy); raw twin (same loop) {2 * span / tr / 1e9:.1f} GB/s "
+          f"({tm / tr * 100:.1f}%), apointer overhead {ta / tr - 1:+.3f}")
+assert torch.equal(both[span:], both[:span]), "raw twin copy wrong"
 print("device error", ap.ap_last_device_error(c))
 ap.ap_munmap(c, rd)
 ap.ap_munmap(c, rs)
