@@ -108,17 +108,32 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     t_index = time.time() - t0
     nb = (cfg["W"] // 32) * (cfg["H"] // 32)
     from paper_conf_isca_shaharbs16_b200 import mgpu
-    b0, b1 = mgpu.block_range(nb, rank, world)
+    # N > 1: AP_SCHED_TABLE splits the (table, bucket)-sorted units (each
+    # bucket read by one rank, winners MIN-reduced); the other schedules split
+    # the image into block ranges (winners gathered)
+    bucket = args.schedule == 2 and world > 1
+    if bucket:
+        b0, b1 = 0, nb
+        u0, u1 = mgpu.unit_range(cfg["L"] * nb, rank, world)
+    else:
+        b0, b1 = mgpu.block_range(nb, rank, world)
+        u0, u1 = 0, 0
     tgt_host = torch.from_numpy(img).pin_memory()
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0,
-                        schedule=args.schedule)
+                        schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0)
+
+    def combine():
+        if bucket:
+            return mgpu.reduce_winners_min(win, rank, world, dist)  # one NCCL reduce (S12)
+        return mgpu.gather_winners(win, rank, world, dist, nb)  # one NCCL gather (S12)
+
     def step():
         ap.ap_collage_run(cache, region, inp, win, stream)
         if world > 1:
-            mgpu.gather_winners(win, rank, world, dist, nb)  # one NCCL gather (S12)
+            combine()
 
     link = host_link_peak(torch, dev)
     for _ in range(args.warmup):
@@ -139,7 +154,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     got = win.cpu().numpy().view(np.uint32).copy()
     # the other schedules, for comparison (cold cache, same winners)
     other_res = []
-    for other in (s for s in (0, 1, 2) if s != args.schedule):
+    for other in (s for s in (0, 1, 2) if s != args.schedule and world == 1):
         inp_o = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                               cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
                               block_count=b1 - b0, schedule=other)
@@ -221,14 +236,18 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         e2e.append(s.elapsed_time(e) * 1e-3)
     cands = None
     res = dict(cfg=cfg, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
+               units=(u0, u1), bucket=bucket,
                other=other_res,
                link=link, raw=raw, e2e=e2e, clocks=clk.summary(), t_gen=t_gen, t_pin=t_pin,
                t_index=t_index, h2d=int(tgt_host.numel()), d2h=int(win.numel() * 4),
                is_copy=is_copy, src=src, cands=cands)
     # parity sample vs the oracle (rank 0): all blocks for c4, a sample for c5
     res["parity"] = None
-    # the gathered answer (N > 1): every rank's range arrives on rank 0
-    full = mgpu.gather_winners(win, rank, world, dist, nb) if world > 1 else None
+    # the combined answer (N > 1) on rank 0
+    full = combine() if world > 1 else None
+    if bucket and rank == 0:
+        got = full.cpu().numpy().view(np.uint32).copy()  # rank 0's own array is partial
+        res["got"] = got
     if rank == 0 and full is not None and not args.no_cpu_baseline:
         import oracle
         fw = full.cpu().numpy().view(np.uint32)
@@ -242,7 +261,8 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
                                   cfg["N"], o_off, o_ids, b0=rb0, nb=k,
                                   threads=os.cpu_count() or 1)
             ok = ok and bool(np.array_equal(want, fw[rb0:rb0 + k]))
-        res["gathered_parity"] = dict(ranks=world, blocks_per_rank=16, equal=ok)
+        res["gathered_parity"] = dict(ranks=world, blocks_per_rank=16, equal=ok,
+                                      partition="buckets (units)" if bucket else "blocks")
     if rank == 0 and not args.no_cpu_baseline:
         import oracle
         o_off = off.cpu().numpy().view(np.uint32)
@@ -296,8 +316,12 @@ def emit_collage(args, res_all, world, METRIC):
                    "group": args.group,
                    "schedule": SCHED_NAMES[args.schedule],
                    "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",
-                   "parallelism": f"blocks partitioned over {world} rank(s) + NCCL gather"},
-        "collage": {"blocks_rank0": r0["b1"] - r0["b0"], "major_faults": st["major"],
+                   "parallelism": (f"(table, bucket) units partitioned over {world} ranks + NCCL "
+                                   "MIN reduce" if r0.get("bucket") else
+                                   f"blocks partitioned over {world} rank(s) + NCCL gather")},
+        "collage": {"blocks_rank0": r0["b1"] - r0["b0"],
+                    "units_rank0": (r0["units"][1] - r0["units"][0]) if r0.get("bucket") else None,
+                    "major_faults": st["major"],
                     "minor_faults": st["minor"], "evictions": st["evictions"],
                     "fill_GB": round(fill / 1e9, 3), "waits": st["waits"],
                     "device_error": r0["err"], "setup_s": {"generate": round(r0["t_gen"], 2),

@@ -292,6 +292,13 @@ typedef struct {
                                   * bucket runs together; the block's winner is   *
                                   * the atomic 64-bit min over its L units.       *
                                   * Results are identical (per-block argmin).     */
+    /* AP_SCHED_TABLE only: run the slice [unit_begin, unit_begin + unit_count)
+     * of the L * block_count units in (table, bucket) order (unit_count 0 =
+     * all).  Blocks whose units are not all in the slice keep a partial
+     * minimum or the sentinel: ranks that split the units combine their
+     * winners with an unsigned 64-bit MIN reduction (multi-GPU, §8(e)). */
+    uint64_t unit_begin;
+    uint64_t unit_count;
 } ap_collage_in;
 
 #define AP_SCHED_NATURAL 0

@@ -43,7 +43,7 @@ class ap_collage_in(ctypes.Structure):
                 ("bucket_bits", u32), ("w", i32), ("proj_dev", vp), ("bias_dev", vp),
                 ("offsets_dev", vp), ("ids_dev", vp), ("N", u64), ("rec_stride", u32),
                 ("group", u32), ("block_begin", u64), ("block_count", u64), ("mode", i32),
-                ("raw_base", vp), ("schedule", i32)]
+                ("raw_base", vp), ("schedule", i32), ("unit_begin", u64), ("unit_count", u64)]
 
 
 class ap_compute_cfg(ctypes.Structure):

@@ -1,7 +1,15 @@
-"""Multi-GPU collage plumbing: query blocks are split
-into contiguous row-major ranges, one per rank (blocks are independent,
-PAPER.md:419), and the per-block winners are collected on rank 0 with one
-gather (NCCL over NVLink on GPUs; gloo in the CPU tests).  Marshalling only.
+"""Multi-GPU collage plumbing.  Two partitions:
+
+* by image: query blocks are split into contiguous row-major ranges, one per
+  rank (blocks are independent), and the per-block winners are
+  collected on rank 0 with one gather;
+* by bucket (AP_SCHED_TABLE): the L * B (block, table) units, in (table,
+  bucket) order, are split into contiguous ranges, so each LSH bucket -- and
+  the records it lists -- is read by one rank; a block's units may land on
+  several ranks, so the winners are combined with one MIN reduction of the
+  64-bit (dist << 32 | idx) words (R-A3's lexicographic order).
+
+NCCL over NVLink on GPUs; gloo in the CPU tests.  Marshalling only.
 """
 
 
@@ -31,3 +39,27 @@ def gather_winners(win, rank, world, dist, nblocks, dst=0):
         b0, b1 = block_range(nblocks, r, world)
         parts.append(bufs[r][:b1 - b0])
     return torch.cat(parts)
+
+
+def unit_range(nunits, rank, world):
+    """Contiguous range [u0, u1) of the sorted units for rank `rank`."""
+    return rank * nunits // world, (rank + 1) * nunits // world
+
+
+def reduce_winners_min(win, rank, world, dist, dst=0):
+    """Combine per-rank partial winners (int32 [B, 2] = (idx, dist) words, the
+    empty sentinel 0xFFFFFFFF where a rank saw no candidate) into the
+    lexicographic (dist, idx) minimum on `dst`; returns it there, None
+    elsewhere.  The pair read as one little-endian u64 is dist << 32 | idx;
+    flipping its sign bit maps unsigned order onto int64 order, so one
+    signed MIN reduction does it."""
+    import torch
+    if world == 1:
+        return win
+    dev = win.device if dist.get_backend() == "nccl" else "cpu"
+    flip = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
+    w64 = win.to(dev).contiguous().view(torch.int64).view(-1) ^ flip
+    dist.reduce(w64, dst=dst, op=dist.ReduceOp.MIN)
+    if rank != dst:
+        return None
+    return (w64 ^ flip).view(torch.int32).view(-1, 2)

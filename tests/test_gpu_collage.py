@@ -9,6 +9,7 @@ import torch
 import oracle
 import synth
 from helpers import check_invariants, make_records
+from paper_conf_isca_shaharbs16_b200 import mgpu
 
 pytestmark = pytest.mark.gpu
 
@@ -111,6 +112,48 @@ def test_collage_partitioned_blocks_equal_whole(ap):
                                                       schedule=g % 3), part)
             parts.append(part)
         assert torch.equal(torch.cat(parts), full)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_collage_unit_slices_min_reduce_to_whole(ap, world):
+    """The bucket partition (mgpu.unit_range + reduce_winners_min) on one GPU:
+    each slice of the (table, bucket)-sorted units runs alone into its own
+    winners array; the unsigned 64-bit MIN over the slices equals the single
+    run and the oracle."""
+    dev = torch.device("cuda:0")
+    n, stride, w, bb, L, K = 2048, 4096, 2500, 8, 4, 5
+    W, H = 256, 192
+    recs, proj, bias, img, *_ = _setup(n, W, H, L, K, w, bb, seed=6)
+    cache = ap.ap_cache_create(90, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        full = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                  group=8), full)
+        flip = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
+        acc = None
+        for g in range(world):
+            u0, u1 = mgpu.unit_range(L * nb, g, world)
+            part = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+            ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                      group=8, unit_begin=u0,
+                                                      unit_count=u1 - u0), part)
+            f = part.view(torch.int64).view(-1) ^ flip
+            acc = f if acc is None else torch.minimum(acc, f)
+        got = (acc ^ flip).view(torch.int32).view(-1, 2)
+        torch.cuda.synchronize()
+        assert ap.ap_last_device_error(cache) == 0
+        assert torch.equal(got, full)
+        o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+        assert np.array_equal(got.cpu().numpy().view(np.uint32), want)
+        assert check_invariants(ap, cache, [r], 90) == []
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)

@@ -72,3 +72,50 @@ def test_block_ranges_cover_exactly():
             assert rs[0][0] == 0 and rs[-1][1] == nb
             assert all(rs[i][1] == rs[i + 1][0] for i in range(world - 1))
             assert max(b - a for a, b in rs) - min(b - a for a, b in rs) <= 1
+
+
+def _worker_tables(rank, world, port, q):
+    """Bucket partition (AP_SCHED_TABLE across ranks): rank r owns the units of
+    tables t = r, r + world, ...; its partial winners (oracle over those
+    tables' buckets only) are combined by the unsigned 64-bit MIN reduction."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, stride, w, bb, recs, proj, bias, img, off, ids = _setup()
+    mine_off = off.copy()
+    for t in range(off.shape[0]):
+        if t % world != rank:
+            mine_off[t] = 0  # every bucket of a table this rank does not own is empty
+    part = oracle.collage(img, proj, bias, w, bb, recs, stride, n, mine_off, ids, threads=1)
+    full = mgpu.reduce_winners_min(torch.from_numpy(part.view(np.int32).copy()), rank, world, dist)
+    if rank == 0:
+        q.put(full.numpy().view(np.uint32).copy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_bucket_partition_min_reduces_to_the_whole_answer(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_tables, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    n, stride, w, bb, recs, proj, bias, img, off, ids = _setup()
+    want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, off, ids, threads=1)
+    assert np.array_equal(got, want)
+    # some block must have had candidates in only part of the tables, else
+    # the reduction was not exercised
+    assert (want[:, 0] != 0xFFFFFFFF).any()
+
+
+def test_unit_ranges_cover_exactly():
+    for nu in (1, 9, 4096, 262144):
+        for world in (1, 2, 3, 8):
+            rs = [mgpu.unit_range(nu, r, world) for r in range(world)]
+            assert rs[0][0] == 0 and rs[-1][1] == nu
+            assert all(rs[i][1] == rs[i + 1][0] for i in range(world - 1))

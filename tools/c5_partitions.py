@@ -1,12 +1,15 @@
 """C5 partitions on one GPU: the collage's query blocks are
-split into G contiguous ranges (mgpu.block_range, as bench.py --gpus G does),
-and each rank's range is run ALONE on this GPU from a cold 2 GiB cache.  With
+split into G contiguous ranges (mgpu.block_range), or -- with AP_SCHED_TABLE,
+as bench.py --gpus G does -- the (table, bucket)-sorted units are
+(mgpu.unit_range), and each rank's share is run ALONE on this GPU from a cold
+2 GiB cache.  With
 G GPUs each rank has its own page cache and its own host link, so the G-GPU
 step time is max over ranks of these per-range times, provided the host's
 memory system feeds G links at once (not measured here: one GPU per call).
 Prints, per G: per-rank seconds, fills, and max / (T1 / G).
 
-Usage: python tools/c5_partitions.py [schedule]     (default 2 = AP_SCHED_TABLE)"""
+Usage: python tools/c5_partitions.py [schedule] [blocks|units]
+       (default: schedule 2 = AP_SCHED_TABLE, partitioned by units)"""
 import os
 import sys
 
@@ -41,10 +44,10 @@ nb = (cfg["W"] // 32) * (cfg["H"] // 32)
 full = None
 
 
-def run_range(b0, b1, reps=2):
+def run_range(b0, b1, reps=2, u0=0, u1=0):
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=8, block_begin=b0, block_count=b1 - b0,
-                        schedule=sched)
+                        schedule=sched, unit_begin=u0, unit_count=u1 - u0)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     ts = []
     for _ in range(reps):
@@ -59,18 +62,30 @@ def run_range(b0, b1, reps=2):
     return min(ts), ap.ap_cache_stats(cache)["fill_bytes"], win
 
 
-print(f"# C5 block ranges run alone on one B200 (cold 2 GiB cache each), schedule {sched}; "
-      f"{nb} blocks, {cfg['N']} records")
+mode = sys.argv[2] if len(sys.argv) > 2 else ("units" if sched == 2 else "blocks")
+print(f"# C5 partitions run alone on one B200 (cold 2 GiB cache each), schedule {sched}, "
+      f"partition by {mode}; {nb} blocks, {cfg['N']} records")
+flip = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
 t1 = None
 for G in (1, 2, 4, 8):
     per, fills, parts = [], [], []
     for r in range(G):
-        b0, b1 = mgpu.block_range(nb, r, G)
-        t, fb, w = run_range(b0, b1)
+        if mode == "units":  # rank r: a slice of the (table, bucket)-sorted units, all blocks
+            u0, u1 = mgpu.unit_range(cfg["L"] * nb, r, G)
+            t, fb, w = run_range(0, nb, u0=u0, u1=u1)
+        else:
+            b0, b1 = mgpu.block_range(nb, r, G)
+            t, fb, w = run_range(b0, b1)
         per.append(t)
         fills.append(fb)
         parts.append(w)
-    whole = torch.cat(parts)
+    if mode == "units":  # the MIN reduction of reduce_winners_min, on one device
+        acc = parts[0].view(torch.int64).view(-1) ^ flip
+        for w in parts[1:]:
+            acc = torch.minimum(acc, w.view(torch.int64).view(-1) ^ flip)
+        whole = (acc ^ flip).view(torch.int32).view(-1, 2)
+    else:
+        whole = torch.cat(parts)
     if full is None:
         full = whole
     same = bool(torch.equal(whole, full))
