@@ -128,18 +128,22 @@ constexpr int STAT_SHARDS = 64;
 
 struct dev_cache;
 
-/* Region descriptor (one mapped file), 64-B aligned in device memory. */
-struct alignas(64) dev_region {
-    const uint8_t* host;    /* device alias of the pinned host bytes      */
+/* Region descriptor (one mapped file), 128-B aligned in device memory.  The
+ * first 64 B hold everything a link or an unlink reads (one sector fetch
+ * after an acquire has invalidated L1; no dependent pointer chase to the
+ * cache descriptor on the minor-fault path). */
+struct alignas(128) dev_region {
     uint64_t bytes;         /* file size                                  */
-    uint64_t npages;        /* ceil(bytes / page)                         */
     uint64_t* pte;          /* npages entries                             */
-    const dev_cache* cache; /* owning cache                               */
-    uint32_t id;            /* region id (< 65535)                        */
-    uint32_t live;          /* 1 while mapped                             */
     const uint8_t* pool;    /* the cache's frame pool (one hop for links) */
+    dev_stats* stats;       /* the cache's counter shards                 */
+    uint32_t id;            /* region id (< 65535)                        */
     uint32_t prot;          /* PROT_READ | PROT_WRITE                     */
+    uint32_t live;          /* 1 while mapped                             */
     uint32_t pad_;
+    const uint8_t* host;    /* device alias of the pinned host bytes      */
+    uint64_t npages;        /* ceil(bytes / page)                         */
+    const dev_cache* cache; /* owning cache                               */
 };
 
 /* Cache descriptor, one copy in device memory per ap_cache_t. */
@@ -318,7 +322,7 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
         printf("[unlink] w%u m%08x grp%08x n%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, grp, n, (unsigned long long)page);
 #endif
         red_add_release(r->pte + page, (uint64_t)0 - (uint64_t)n);
-        stat_add(&my_stats(r->cache)->unlinks, 1);
+        stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->unlinks, 1);
     }
 }
 
@@ -725,7 +729,7 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
     }
     const unsigned linkedm = __ballot_sync(m, is_leader && (old >> 62) == 2);
     if (linkedm && (int)lane_id() == __ffs(m) - 1)
-        stat_add(&my_stats(r->cache)->minor, __popc(linkedm));
+        stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->minor, __popc(linkedm));
     old = __shfl_sync(m, old, leader);
     const bool ok = !need || (old >> 62) == 2;
     if (need && ok) {

@@ -298,6 +298,7 @@ extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, 
     d.pte = rg.pte;
     d.cache = c->d_cache;
     d.pool = c->pool;
+    d.stats = c->stats;
     d.prot = (uint32_t)prot;
     d.id = id;
     d.live = 1;
