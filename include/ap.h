@@ -99,6 +99,45 @@ int ap_msync(ap_cache_t cache, ap_region_t region);
  * (a linked apointer). */
 int ap_munmap(ap_cache_t cache, ap_region_t region);
 
+/* ------------------------------------------ peer page caches (NEXT N2)
+ * SURVEY 8(f) N2; PAPER.md:33 names distributed shared memory across GPUs as
+ * a motivation.  Several caches (typically one per GPU) may map the same
+ * file.  Declaring another cache's region as a peer of `region` makes a
+ * major fault first look the page up in the peer's page table and, if it is
+ * resident there, copy the peer's frame (HBM-to-HBM over NVLink 5 / the same
+ * HBM) instead of reading the page over the host link; the peer's page is
+ * pinned by its reference count during the copy, so the peer
+ * can keep running and evicting.  Both mappings must be read-only, have the
+ * same size and the same page size.  Up to 7 peers per region, tried in the
+ * order added.  The caller keeps every peer mapped (and its cache alive)
+ * until ap_region_clear_peers (or ap_munmap) of `region` returns.
+ * Errors: AP_EINVAL (mismatch, writable, peer == cache, GPUs without peer
+ * access), AP_ERANGE (7 peers already), AP_ECUDA. */
+
+/* Same process: `peer_region` of `peer` (any GPU with peer access to this
+ * cache's GPU, or the same GPU). */
+int ap_region_add_peer(ap_cache_t cache, ap_region_t region, ap_cache_t peer,
+                       ap_region_t peer_region);
+
+/* Across processes (one process per GPU): ap_region_export writes a plain
+ * byte record (CUDA IPC handles of the region's page table and of the frame
+ * pool, plus sizes) that another process passes to ap_region_add_peer_ipc,
+ * e.g. after an all-gather over torch.distributed.  The exporting process
+ * keeps the cache and region alive until the importers cleared their peers. */
+typedef struct {
+    uint8_t pte_handle[64];  /* cudaIpcMemHandle_t of the PTE array          */
+    uint8_t pool_handle[64]; /* cudaIpcMemHandle_t of the frame pool block   */
+    uint64_t pool_offset;    /* frame pool start inside that block           */
+    uint64_t bytes;          /* region size                                  */
+    uint32_t page_size;
+    int32_t device;          /* exporter's device ordinal (informational)    */
+} ap_peer_handle_t;
+int ap_region_export(ap_cache_t cache, ap_region_t region, ap_peer_handle_t* out);
+int ap_region_add_peer_ipc(ap_cache_t cache, ap_region_t region, const ap_peer_handle_t* h);
+
+/* Forget every peer of `region` (and close the IPC mappings); synchronises. */
+int ap_region_clear_peers(ap_cache_t cache, ap_region_t region);
+
 /* Device-accessible alias of the region's host bytes (the zero-copy view the
  * fault path fills from). Useful for raw-pointer twins. */
 int ap_region_devptr(ap_cache_t cache, ap_region_t region, const void** out);
@@ -113,6 +152,8 @@ typedef struct {
     uint64_t downgrades;  /* lanes proactively unlinked under frame pressure      */
     uint64_t nofree;      /* allocation attempts that found no evictable frame    */
     uint64_t unlinks;     /* warp-aggregated reference-count decrements           */
+    uint64_t peer_fills;  /* major faults served from a peer cache (N2)           */
+    uint64_t peer_bytes;  /* bytes those fills copied from peer frames            */
 } ap_stats_t;
 
 /* Sum of the device counters since create/reset (synchronises the device). */

@@ -123,10 +123,20 @@ constexpr int POLICY_RANDOM = 1;
 /* Counters, sharded by SM to keep atomics off one address. */
 struct alignas(64) dev_stats {
     unsigned long long major, minor, fill_bytes, evictions, waits, downgrades, nofree, unlinks;
+    unsigned long long peer_fills, peer_bytes; /* N2: fills copied from a peer cache */
 };
 constexpr int STAT_SHARDS = 64;
 
 struct dev_cache;
+
+/* A peer page cache holding the same file (NEXT N2): its
+ * region's page table and its frame pool, as addresses this GPU can read
+ * (the same HBM, NVLink peer access, or a CUDA IPC mapping of them). */
+struct dev_peer {
+    uint64_t* pte;       /* the peer region's PTE array (same page numbers) */
+    const uint8_t* pool; /* the peer cache's frame pool                     */
+};
+constexpr uint32_t MAX_PEERS = 7;
 
 /* Region descriptor (one mapped file), 128-B aligned in device memory.  The
  * first 64 B hold everything a link or an unlink reads (one sector fetch
@@ -144,6 +154,8 @@ struct alignas(128) dev_region {
     const uint8_t* host;    /* device alias of the pinned host bytes      */
     uint64_t npages;        /* ceil(bytes / page)                         */
     const dev_cache* cache; /* owning cache                               */
+    const dev_peer* peers;  /* N2: caches a major fault may copy from     */
+    uint32_t npeers;        /* 0 = fills come from the host only          */
 };
 
 /* Cache descriptor, one copy in device memory per ap_cache_t. */
@@ -238,6 +250,43 @@ __device__ __forceinline__ uint64_t add_acquire(uint64_t* p, uint64_t v) {
                  : "=l"(old) : "l"(p), "l"(v) : "memory");
     return old;
 }
+/* Link / unlink RMWs on a PTE.  AP_LINK_RELAXED: the link add is relaxed;
+ * frame data is read with .cg loads whose address is computed from the add's
+ * result (ablation).  AP_UNLINK_RELAXED: relaxed unlink (measurement only:
+ * bounds what the release costs; not safe against eviction). */
+__device__ __forceinline__ uint64_t add_link(uint64_t* p, uint64_t v) {
+#ifdef AP_LINK_RELAXED
+    uint64_t old;
+    asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;"
+                 : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+#else
+    return add_acquire(p, v);
+#endif
+}
+__device__ __forceinline__ void red_unlink(uint64_t* p, uint64_t v) {
+#ifdef AP_UNLINK_RELAXED
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+#else
+    red_add_release(p, v);
+#endif
+}
+/* System-scope RMWs on a peer's PTE: the peer's own warps update it from
+ * their GPU, so these are performed at the peer's memory with .sys scope. */
+__device__ __forceinline__ uint64_t ld_relaxed_sys(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t add_acquire_sys(uint64_t* p, uint64_t v) {
+    uint64_t old;
+    asm volatile("atom.acquire.sys.global.add.u64 %0, [%1], %2;"
+                 : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ void red_add_release_sys(uint64_t* p, uint64_t v) {
+    asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void red_add_relaxed(unsigned long long* p, unsigned long long v) {
     asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -321,7 +370,7 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
 #ifdef AP_DEBUG
         printf("[unlink] w%u m%08x grp%08x n%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, grp, n, (unsigned long long)page);
 #endif
-        red_add_release(r->pte + page, (uint64_t)0 - (uint64_t)n);
+        red_unlink(r->pte + page, (uint64_t)0 - (uint64_t)n);
         stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->unlinks, 1);
     }
 }
@@ -496,6 +545,62 @@ __device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, const 
     }
 }
 
+/* -------------------------------------------------------------------------
+ * N2 peer fill (the "distributed shared memory across GPUs"
+ * motivation of PAPER.md:33): before going to the host link, the warp looks
+ * for page `pg` in the peer caches mapped over the same file.  The first
+ * lane reads the peer's PTE; if it is VALID it pins the page there with one
+ * acquire add (the peer cannot evict a frame whose count is positive,
+ * PAPER.md:145), the warp copies the frame (HBM or NVLink instead of PCIe),
+ * and the pin is dropped with a release add once every lane's loads are done
+ * (each load feeds a store, and __syncwarp orders the lanes before the
+ * leader's release).  Returns false, having copied nothing, when no peer has
+ * the page resident.  The peer frame already holds a ragged last page
+ * zero-padded, so the whole frame is copied. */
+static __device__ __noinline__ bool fill_from_peer(unsigned m, const dev_cache* c, const dev_region* r,
+                                            uint64_t f, uint64_t pg) {
+    const unsigned first = __ffs(m) - 1;
+    const unsigned lane = lane_id();
+    const unsigned rk = __popc(m & lanemask_lt());
+    const unsigned nl = __popc(m);
+    const uint64_t P = 1ull << c->log2_page;
+    for (uint32_t i = 0; i < r->npeers; ++i) {
+        const dev_peer pr = r->peers[i];
+        uint64_t* q = pr.pte + pg;
+        uint64_t old = 0;
+        if (lane == first && (ld_relaxed_sys(q) >> 62) == 2) {
+            old = add_acquire_sys(q, 1);
+            if ((old >> 62) != 2) {
+                red_add_release_sys(q, (uint64_t)0 - 1); /* transient count, undone */
+                old = 0;
+            }
+        }
+        old = __shfl_sync(m, old, first);
+        if ((old >> 62) != 2) continue;
+        const uint4* s4 = reinterpret_cast<const uint4*>(pr.pool + ((old >> 32) & PTE_FRAME_MASK) * P);
+        uint4* d4 = reinterpret_cast<uint4*>(c->pool + f * P);
+        const uint64_t nvec = P / 16;
+        constexpr int U = 8;
+        for (uint64_t j = rk; j < nvec; j += (uint64_t)nl * U) {
+            uint4 v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (j + (uint64_t)nl * u < nvec) v[u] = __ldcg(s4 + j + (uint64_t)nl * u);
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (j + (uint64_t)nl * u < nvec) __stcg(d4 + j + (uint64_t)nl * u, v[u]);
+        }
+        __syncwarp(m);
+        if (lane == first) {
+            red_add_release_sys(q, (uint64_t)0 - 1);
+            stat_add(&my_stats(c)->peer_fills, 1);
+            stat_add(&my_stats(c)->peer_bytes, P);
+        }
+        return true;
+    }
+    return false;
+}
+
 template <class T>
 struct slow_out {
     uint64_t x;
@@ -554,7 +659,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
          * add is undone.  Every other transition tolerates such transient
          * counts on non-VALID entries: publish and revert are adds, claims
          * are CASes from exactly EMPTY (R-A17). */
-        uint64_t old = is_leader ? add_acquire(pte, n) : 0;
+        uint64_t old = is_leader ? add_link(pte, n) : 0;
 #ifdef AP_DEBUG
         if (is_leader && (old >> 62) == 2) printf("[link] w%u m%08x n%u pg %llu old %llx\n", (unsigned)(threadIdx.x >> 5), m, n, (unsigned long long)pg, (unsigned long long)old);
 #endif
@@ -610,8 +715,9 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             const dev_region* fr =
                 reinterpret_cast<const dev_region*>(__shfl_sync(m, (unsigned long long)r, L));
             if ((int)lane == L) st_relaxed(c->owner + f, ((uint64_t)(fr->id + 1) << 48) | fpg);
-            fill_page(m, c, fr, f, fpg);
-            if ((int)lane == __ffs(m) - 1) {
+            const bool from_peer = fr->npeers && fill_from_peer(m, c, fr, f, fpg);
+            if (!from_peer) fill_page(m, c, fr, f, fpg);
+            if (!from_peer && (int)lane == __ffs(m) - 1) {
                 const uint64_t avail = fr->bytes - (fpg << lg);
                 stat_add(&S->fill_bytes, avail < P ? avail : P);
             }
@@ -719,7 +825,7 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
     uint64_t old = 0;
     if (is_leader) {
         uint64_t* pte = r->pte + pg;
-        old = add_acquire(pte, __popc(grp));
+        old = add_link(pte, __popc(grp));
         if ((old >> 62) == 2) {
             if (!(old & PTE_REF)) red_or_relaxed(pte, PTE_REF);
         } else {

@@ -102,6 +102,30 @@ def ap_region_devptr(cache, region):
     return p.value
 
 
+def ap_region_add_peer(cache, region, peer, peer_region):
+    """N2: major faults of `region` copy pages resident in `peer_region` of
+    the cache `peer` (same process; same or peer-accessible GPU)."""
+    _lib.check("ap_region_add_peer", _lib.lib().ap_region_add_peer(cache, region, peer, peer_region))
+
+
+def ap_region_export(cache, region):
+    """N2 across processes: the region's peer record as bytes (CUDA IPC
+    handles + sizes), to hand to ap_region_add_peer_ipc in another process."""
+    h = _lib.ap_peer_handle_t()
+    _lib.check("ap_region_export", _lib.lib().ap_region_export(cache, region, ctypes.byref(h)))
+    return bytes(h)
+
+
+def ap_region_add_peer_ipc(cache, region, handle):
+    h = _lib.ap_peer_handle_t.from_buffer_copy(bytes(handle))
+    _lib.check("ap_region_add_peer_ipc",
+               _lib.lib().ap_region_add_peer_ipc(cache, region, ctypes.byref(h)))
+
+
+def ap_region_clear_peers(cache, region):
+    _lib.check("ap_region_clear_peers", _lib.lib().ap_region_clear_peers(cache, region))
+
+
 def ap_region_npages(cache, region):
     n = ctypes.c_uint64()
     _lib.check("ap_region_npages", _lib.lib().ap_region_npages(cache, region, ctypes.byref(n)))

@@ -25,10 +25,16 @@ u64, u32, i32, vp, ci = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes
 
 class ap_stats_t(ctypes.Structure):
     _fields_ = [(n, u64) for n in ("major", "minor", "fill_bytes", "evictions", "waits",
-                                   "downgrades", "nofree", "unlinks")]
+                                   "downgrades", "nofree", "unlinks", "peer_fills",
+                                   "peer_bytes")]
 
     def as_dict(self):
         return {n: int(getattr(self, n)) for n, _ in self._fields_}
+
+
+class ap_peer_handle_t(ctypes.Structure):
+    _fields_ = [("pte_handle", ctypes.c_uint8 * 64), ("pool_handle", ctypes.c_uint8 * 64),
+                ("pool_offset", u64), ("bytes", u64), ("page_size", u32), ("device", i32)]
 
 
 class ap_bench_cfg(ctypes.Structure):
@@ -96,6 +102,10 @@ def lib():
             "ap_msync": (ci, [vp, u32]),
             "ap_bench_write": (ci, [vp, u32, ctypes.POINTER(ap_bench_cfg), vp]),
             "ap_bench_copy": (ci, [vp, u32, u32, ctypes.POINTER(ap_bench_cfg), vp]),
+            "ap_region_add_peer": (ci, [vp, u32, vp, u32]),
+            "ap_region_export": (ci, [vp, u32, ctypes.POINTER(ap_peer_handle_t)]),
+            "ap_region_add_peer_ipc": (ci, [vp, u32, ctypes.POINTER(ap_peer_handle_t)]),
+            "ap_region_clear_peers": (ci, [vp, u32]),
             "ap_lsh_build_index": (ci, [vp, u32, u64, u32, u32, u32, u32, i32, vp, vp, vp, vp,
                                         vp]),
         }
@@ -113,7 +123,8 @@ EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", 
             "ap_last_device_error", "ap_cache_dump", "ap_region_dump_pte", "ap_prefill",
             "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index",
             "ap_bench_latency", "ap_mmap_prot", "ap_msync", "ap_bench_write", "ap_bench_copy",
-            "ap_bench_compute", "ap_cache_set_backoff"]
+            "ap_bench_compute", "ap_cache_set_backoff", "ap_region_add_peer", "ap_region_export",
+            "ap_region_add_peer_ipc", "ap_region_clear_peers"]
 
 
 def check(fn, rc):

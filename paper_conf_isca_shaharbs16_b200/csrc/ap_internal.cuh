@@ -22,6 +22,9 @@ struct ap_region_host {
     bool registered = false; /* we called cudaHostRegister                 */
     bool live = false;
     uint32_t prot = 1;       /* AP_PROT_*                                  */
+    std::vector<ap::dev_peer> peers;  /* N2 peer caches (device-readable)  */
+    ap::dev_peer* d_peers = nullptr;  /* their device copy                 */
+    std::vector<void*> ipc_opened;    /* CUDA IPC mappings to close        */
 };
 
 struct ap_cache_s {

@@ -4,6 +4,7 @@
  * statistics, reset, dumps, prefill.  C ABI in include/ap.h.
  */
 #include <cuda_runtime.h>
+#include <cstring>
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
@@ -326,6 +327,12 @@ extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
     if (!ap_region_ok(c, r)) return AP_EINVAL;
     ap_device_guard g(c->device);
     AP_CUDA_TRY(cudaDeviceSynchronize());
+    if (!c->reg[r].peers.empty() || c->reg[r].d_peers) {
+        int rcp = ap_region_clear_peers(c, r);
+        if (rcp) return rcp;
+        cudaFree(c->reg[r].d_peers);
+        c->reg[r].d_peers = nullptr;
+    }
     if (c->reg[r].prot & AP_PROT_WRITE) {
         int rc0 = ap_msync(c, r);
         if (rc0) return rc0;
@@ -344,6 +351,109 @@ extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
     cudaFree(rg.pte);
     if (rg.registered) cudaHostUnregister(const_cast<void*>(rg.host_buf));
     rg = ap_region_host{};
+    return AP_OK;
+}
+
+/* ------------------------------------------------------------ N2 peers */
+static int push_region_peers(ap_cache_s* c, ap_region_t r) {
+    ap_region_host& rg = c->reg[r];
+    if (!rg.d_peers && cudaMalloc(&rg.d_peers, sizeof(ap::dev_peer) * ap::MAX_PEERS) != cudaSuccess) {
+        cudaGetLastError();
+        return AP_ENOMEM;
+    }
+    if (!rg.peers.empty())
+        AP_CUDA_TRY(cudaMemcpy(rg.d_peers, rg.peers.data(), sizeof(ap::dev_peer) * rg.peers.size(),
+                               cudaMemcpyHostToDevice));
+    ap::dev_region d{};
+    AP_CUDA_TRY(cudaMemcpy(&d, c->regions + r, sizeof d, cudaMemcpyDeviceToHost));
+    d.peers = rg.d_peers;
+    d.npeers = (uint32_t)rg.peers.size();
+    AP_CUDA_TRY(cudaMemcpy(c->regions + r, &d, sizeof d, cudaMemcpyHostToDevice));
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    return AP_OK;
+}
+
+static int peer_compatible(const ap_cache_s* c, ap_region_t r, uint32_t page, uint64_t bytes) {
+    const ap_region_host& rg = c->reg[r];
+    if (page != c->page || bytes != rg.bytes) return AP_EINVAL;
+    if (rg.prot & AP_PROT_WRITE) return AP_EINVAL;
+    if (rg.peers.size() >= ap::MAX_PEERS) return AP_ERANGE;
+    return AP_OK;
+}
+
+extern "C" int ap_region_add_peer(ap_cache_t c, ap_region_t r, ap_cache_t pc, ap_region_t pr) {
+    if (!ap_region_ok(c, r) || !ap_region_ok(pc, pr) || c == pc) return AP_EINVAL;
+    if (pc->reg[pr].prot & AP_PROT_WRITE) return AP_EINVAL;
+    int rc = peer_compatible(c, r, pc->page, pc->reg[pr].bytes);
+    if (rc) return rc;
+    ap_device_guard g(c->device);
+    if (pc->device != c->device) {
+        int ok = 0;
+        AP_CUDA_TRY(cudaDeviceCanAccessPeer(&ok, c->device, pc->device));
+        if (!ok) return AP_EINVAL;
+        cudaError_t e = cudaDeviceEnablePeerAccess(pc->device, 0);
+        if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+        else AP_CUDA_TRY(e);
+    }
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    c->reg[r].peers.push_back(ap::dev_peer{pc->reg[pr].pte, pc->pool});
+    return push_region_peers(c, r);
+}
+
+extern "C" int ap_region_export(ap_cache_t c, ap_region_t r, ap_peer_handle_t* out) {
+    if (!ap_region_ok(c, r) || !out) return AP_EINVAL;
+    if (c->reg[r].prot & AP_PROT_WRITE) return AP_EINVAL;
+    static_assert(sizeof(cudaIpcMemHandle_t) <= sizeof out->pte_handle, "IPC handle size");
+    ap_device_guard g(c->device);
+    ap_peer_handle_t h{};
+    cudaIpcMemHandle_t a, b;
+    AP_CUDA_TRY(cudaIpcGetMemHandle(&a, c->reg[r].pte));
+    AP_CUDA_TRY(cudaIpcGetMemHandle(&b, c->pool_raw));
+    memcpy(h.pte_handle, &a, sizeof a);
+    memcpy(h.pool_handle, &b, sizeof b);
+    h.pool_offset = (uint64_t)(c->pool - (uint8_t*)c->pool_raw);
+    h.bytes = c->reg[r].bytes;
+    h.page_size = c->page;
+    h.device = c->device;
+    *out = h;
+    return AP_OK;
+}
+
+extern "C" int ap_region_add_peer_ipc(ap_cache_t c, ap_region_t r, const ap_peer_handle_t* h) {
+    if (!ap_region_ok(c, r) || !h) return AP_EINVAL;
+    int rc = peer_compatible(c, r, h->page_size, h->bytes);
+    if (rc) return rc;
+    ap_device_guard g(c->device);
+    cudaIpcMemHandle_t a, b;
+    memcpy(&a, h->pte_handle, sizeof a);
+    memcpy(&b, h->pool_handle, sizeof b);
+    void* pte = nullptr;
+    void* pool = nullptr;
+    AP_CUDA_TRY(cudaIpcOpenMemHandle(&pte, a, cudaIpcMemLazyEnablePeerAccess));
+    cudaError_t e = cudaIpcOpenMemHandle(&pool, b, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+        cudaIpcCloseMemHandle(pte);
+        AP_CUDA_TRY(e);
+    }
+    ap_region_host& rg = c->reg[r];
+    rg.ipc_opened.push_back(pte);
+    rg.ipc_opened.push_back(pool);
+    rg.peers.push_back(ap::dev_peer{(uint64_t*)pte, (const uint8_t*)pool + h->pool_offset});
+    return push_region_peers(c, r);
+}
+
+extern "C" int ap_region_clear_peers(ap_cache_t c, ap_region_t r) {
+    if (!ap_region_ok(c, r)) return AP_EINVAL;
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    ap_region_host& rg = c->reg[r];
+    rg.peers.clear();
+    if (rg.d_peers) {
+        int rc = push_region_peers(c, r);
+        if (rc) return rc;
+    }
+    for (void* p : rg.ipc_opened) cudaIpcCloseMemHandle(p);
+    rg.ipc_opened.clear();
     return AP_OK;
 }
 
@@ -377,6 +487,8 @@ extern "C" int ap_cache_stats(ap_cache_t c, ap_stats_t* out) {
         t.downgrades += x.downgrades;
         t.nofree += x.nofree;
         t.unlinks += x.unlinks;
+        t.peer_fills += x.peer_fills;
+        t.peer_bytes += x.peer_bytes;
     }
     *out = t;
     return AP_OK;

@@ -27,10 +27,15 @@ def _run(ap, cache, region, cfg, nthreads, dev, out_bytes=None):
     return out.cpu().numpy()
 
 
+ACCESS = [0, 2]  # AP_ACCESS_TILE, AP_ACCESS_RANGE
+
+
+@pytest.mark.parametrize("access", ACCESS)
 @pytest.mark.parametrize("frames", [1, 8, 64, 4096])
 @pytest.mark.parametrize("elem", [4, 16])
-def test_seq_copy_is_the_file(ap, dev, frames, elem):
-    """C1 shape: warps walk pages, every read faults while frames < pages."""
+def test_seq_copy_is_the_file(ap, dev, frames, elem, access):
+    """C1 shape: warps walk pages, every read faults while frames < pages.
+    Both tiled access styles (tiles; one pin per unit) give the file."""
     nbytes = (1 << 20) + 3 * 4096 + 48  # ragged last page
     f = make_file(nbytes, seed=1)
     cache = ap.ap_cache_create(frames, 4096)
@@ -38,7 +43,7 @@ def test_seq_copy_is_the_file(ap, dev, frames, elem):
         r = ap.ap_mmap(cache, f)
         grid, block = (2, 64) if frames == 1 else (8, 128)
         cfg = ap.bench_cfg(ap.AP_SEQ, elem, grid, block, unit_bytes=4096, out_copy=True,
-                           span_bytes=nbytes)
+                           span_bytes=nbytes, access=access)
         out = _run(ap, cache, r, cfg, grid * block, dev, out_bytes=nbytes)
         whole = nbytes // elem * elem
         assert np.array_equal(out[:whole], f[:whole])
@@ -56,7 +61,8 @@ def test_seq_copy_is_the_file(ap, dev, frames, elem):
 
 @pytest.mark.parametrize("elem,unit,passes", [(16, 4096, 1), (16, 16384, 3), (4, 2048, 2),
                                               (8, 65536, 1)])
-def test_seq_checksums(ap, dev, elem, unit, passes):
+@pytest.mark.parametrize("access", ACCESS)
+def test_seq_checksums(ap, dev, elem, unit, passes, access):
     page = 65536
     nbytes = 4 * (1 << 20) + 777 * 16
     f = make_file(nbytes, seed=2)
@@ -65,7 +71,7 @@ def test_seq_checksums(ap, dev, elem, unit, passes):
         r = ap.ap_mmap(cache, f)
         grid, block = 6, 256
         cfg = ap.bench_cfg(ap.AP_SEQ, elem, grid, block, unit_bytes=unit, passes=passes,
-                           span_bytes=nbytes)
+                           span_bytes=nbytes, access=access)
         got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
         want = oracle.read_seq(f, nbytes, unit, elem, grid * block, passes)
         assert np.array_equal(got, want)
