@@ -371,7 +371,9 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
         printf("[unlink] w%u m%08x grp%08x n%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, grp, n, (unsigned long long)page);
 #endif
         red_unlink(r->pte + page, (uint64_t)0 - (uint64_t)n);
+#ifndef AP_NO_HOT_STATS
         stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->unlinks, 1);
+#endif
     }
 }
 
@@ -512,19 +514,17 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
 }
 
 /* -------------------------------------------------------------------------
- * S8 fill: the whole warp copies one page from pinned host memory (over the
- * host link, zero-copy 16-B loads) into frame `f`; a ragged last page is
- * zero-padded.  Host bytes are 16-B aligned (ap_mmap checks it). */
-__device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, const dev_region* r,
-                                          uint64_t f, uint64_t pg) {
+ * S8 fill: the whole warp copies one page into frame `f` with 16-B loads,
+ * from pinned host memory over the host link (zero copy) or, for N2, from a
+ * peer cache's frame; the first `len` bytes come from `src` and a ragged
+ * last page is zero-padded.  Host bytes are 16-B aligned (ap_mmap checks it). */
+__device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, uint64_t f,
+                                          const uint8_t* src, uint64_t len) {
     /* the lanes in m share the copy: rank = position among them */
     const unsigned lane = __popc(m & lanemask_lt());
     const unsigned nl = __popc(m);
     const uint64_t P = 1ull << c->log2_page;
     uint8_t* dst = c->pool + f * P;
-    const uint8_t* src = r->host + pg * P;
-    const uint64_t avail = r->bytes - pg * P;
-    const uint64_t len = avail < P ? avail : P;
     const uint64_t nvec = len / 16;
     const uint4* s4 = reinterpret_cast<const uint4*>(src);
     uint4* d4 = reinterpret_cast<uint4*>(dst);
@@ -539,7 +539,7 @@ __device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, const 
     }
     for (; i < nvec; i += nl) __stcg(d4 + i, __ldcs(s4 + i));
     if (len < P) {
-        /* ragged tail: bytes [nvec*16, len) from host, the rest zeros */
+        /* ragged tail: bytes [nvec*16, len) from the source, the rest zeros */
         for (uint64_t b = nvec * 16 + lane; b < P; b += nl)
             dst[b] = b < len ? src[b] : (uint8_t)0;
     }
@@ -551,24 +551,21 @@ __device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, const 
  * for page `pg` in the peer caches mapped over the same file.  The first
  * lane reads the peer's PTE; if it is VALID it pins the page there with one
  * acquire add (the peer cannot evict a frame whose count is positive,
- * PAPER.md:145), the warp copies the frame (HBM or NVLink instead of PCIe),
- * and the pin is dropped with a release add once every lane's loads are done
- * (each load feeds a store, and __syncwarp orders the lanes before the
- * leader's release).  Returns false, having copied nothing, when no peer has
- * the page resident.  The peer frame already holds a ragged last page
- * zero-padded, so the whole frame is copied. */
-static __device__ __noinline__ bool fill_from_peer(unsigned m, const dev_cache* c, const dev_region* r,
-                                            uint64_t f, uint64_t pg) {
+ * PAPER.md:145).  Returns the pinned peer PTE (and the peer frame in *src),
+ * or nullptr when no peer has the page resident.  The warp then copies the
+ * whole frame (a peer frame holds a ragged last page already zero-padded)
+ * and peer_unpin drops the pin once every lane's loads are done (each load
+ * feeds a store, and __syncwarp orders the lanes before the leader's
+ * release).  Small on purpose: it adds no copy loop to the fault path. */
+__device__ __forceinline__ uint64_t* peer_pin(unsigned m, const dev_cache* c, const dev_region* r,
+                                              uint64_t pg, const uint8_t** src) {
     const unsigned first = __ffs(m) - 1;
-    const unsigned lane = lane_id();
-    const unsigned rk = __popc(m & lanemask_lt());
-    const unsigned nl = __popc(m);
     const uint64_t P = 1ull << c->log2_page;
     for (uint32_t i = 0; i < r->npeers; ++i) {
-        const dev_peer pr = r->peers[i];
-        uint64_t* q = pr.pte + pg;
+        const dev_peer* pr = r->peers + i;
+        uint64_t* q = pr->pte + pg;
         uint64_t old = 0;
-        if (lane == first && (ld_relaxed_sys(q) >> 62) == 2) {
+        if (lane_id() == first && (ld_relaxed_sys(q) >> 62) == 2) {
             old = add_acquire_sys(q, 1);
             if ((old >> 62) != 2) {
                 red_add_release_sys(q, (uint64_t)0 - 1); /* transient count, undone */
@@ -576,29 +573,20 @@ static __device__ __noinline__ bool fill_from_peer(unsigned m, const dev_cache* 
             }
         }
         old = __shfl_sync(m, old, first);
-        if ((old >> 62) != 2) continue;
-        const uint4* s4 = reinterpret_cast<const uint4*>(pr.pool + ((old >> 32) & PTE_FRAME_MASK) * P);
-        uint4* d4 = reinterpret_cast<uint4*>(c->pool + f * P);
-        const uint64_t nvec = P / 16;
-        constexpr int U = 8;
-        for (uint64_t j = rk; j < nvec; j += (uint64_t)nl * U) {
-            uint4 v[U];
-#pragma unroll
-            for (int u = 0; u < U; ++u)
-                if (j + (uint64_t)nl * u < nvec) v[u] = __ldcg(s4 + j + (uint64_t)nl * u);
-#pragma unroll
-            for (int u = 0; u < U; ++u)
-                if (j + (uint64_t)nl * u < nvec) __stcg(d4 + j + (uint64_t)nl * u, v[u]);
+        if ((old >> 62) == 2) {
+            *src = pr->pool + ((old >> 32) & PTE_FRAME_MASK) * P;
+            return q;
         }
-        __syncwarp(m);
-        if (lane == first) {
-            red_add_release_sys(q, (uint64_t)0 - 1);
-            stat_add(&my_stats(c)->peer_fills, 1);
-            stat_add(&my_stats(c)->peer_bytes, P);
-        }
-        return true;
     }
-    return false;
+    return nullptr;
+}
+__device__ __forceinline__ void peer_unpin(unsigned m, const dev_cache* c, uint64_t* q) {
+    __syncwarp(m);
+    if (lane_id() == (unsigned)(__ffs(m) - 1)) {
+        red_add_release_sys(q, (uint64_t)0 - 1);
+        stat_add(&my_stats(c)->peer_fills, 1);
+        stat_add(&my_stats(c)->peer_bytes, 1ull << c->log2_page);
+    }
 }
 
 template <class T>
@@ -715,12 +703,12 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             const dev_region* fr =
                 reinterpret_cast<const dev_region*>(__shfl_sync(m, (unsigned long long)r, L));
             if ((int)lane == L) st_relaxed(c->owner + f, ((uint64_t)(fr->id + 1) << 48) | fpg);
-            const bool from_peer = fr->npeers && fill_from_peer(m, c, fr, f, fpg);
-            if (!from_peer) fill_page(m, c, fr, f, fpg);
-            if (!from_peer && (int)lane == __ffs(m) - 1) {
-                const uint64_t avail = fr->bytes - (fpg << lg);
-                stat_add(&S->fill_bytes, avail < P ? avail : P);
-            }
+                        const uint8_t* src = fr->host + (fpg << lg);
+            const uint64_t avail = fr->bytes - (fpg << lg);
+            uint64_t* peer_q = fr->npeers ? peer_pin(m, c, fr, fpg, &src) : nullptr;
+            fill_page(m, c, f, src, peer_q ? P : (avail < P ? avail : P));
+            if (peer_q) peer_unpin(m, c, peer_q);
+            else if ((int)lane == __ffs(m) - 1) stat_add(&S->fill_bytes, avail < P ? avail : P);
             fence_gpu();
             __syncwarp(m);
 #ifdef AP_DEBUG
@@ -833,9 +821,11 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
                             (unsigned long long)(0 - (uint64_t)__popc(grp)));
         }
     }
+#ifndef AP_NO_HOT_STATS /* ablation: no counters on the inline link / unlink */
     const unsigned linkedm = __ballot_sync(m, is_leader && (old >> 62) == 2);
     if (linkedm && (int)lane_id() == __ffs(m) - 1)
         stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->minor, __popc(linkedm));
+#endif
     old = __shfl_sync(m, old, leader);
     const bool ok = !need || (old >> 62) == 2;
     if (need && ok) {
@@ -1178,7 +1168,7 @@ struct ptr {
         const unsigned m = __activemask();
         const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
         bool ok = linked() && ((x ^ (x + span)) >> lg) == 0;
-        if (!__all_sync(m, ok)) {
+        if (__builtin_expect(!__all_sync(m, ok), 0)) {
             if (__any_sync(m, !linked()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
                 const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
                 x = o.x;
