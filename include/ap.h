@@ -151,7 +151,8 @@ typedef struct {
     uint64_t waits;       /* fault rounds that had to back off                    */
     uint64_t downgrades;  /* lanes proactively unlinked under frame pressure      */
     uint64_t nofree;      /* allocation attempts that found no evictable frame    */
-    uint64_t unlinks;     /* warp-aggregated reference-count decrements           */
+    uint64_t unlinks;     /* warp-aggregated refcount decrements (0 unless the    *
+                           * library is built with -DAP_COUNT_UNLINKS)           */
     uint64_t peer_fills;  /* major faults served from a peer cache (N2)           */
     uint64_t peer_bytes;  /* bytes those fills copied from peer frames            */
 } ap_stats_t;
