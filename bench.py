@@ -512,8 +512,12 @@ def main():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--group", type=int, default=8, help="collage candidates per warp (1, 2, 4, 8)")
-    p.add_argument("--schedule", type=int, default=2, help="collage: 0 = natural, 1 = LSH-sorted blocks, 2 = per-table units")
+    p.add_argument("--schedule", type=int, default=2, help="collage: 0 = natural, 1 = LSH-sorted blocks, 2 = per-table units, 3 = per-table units in bucket-MinHash order")
     p.add_argument("--stride", type=int, default=4096, help="collage record stride (3072 = unaligned)")
+    p.add_argument("--id-chunks", type=int, default=None,
+                   help="collage record-id windows (ap_collage_in.id_chunks; 0 = off; "
+                        "default 8 for c4, 12 for c5: about two windows per cache-full of "
+                        "distinct records)")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     args = p.parse_args()

@@ -19,7 +19,8 @@ import numpy as np
 
 GiB = 1 << 30
 SCHED_NAMES = {0: "natural order (one CTA per block, the paper's single kernel)",
-               1: "lsh-sorted blocks", 2: "per-table units sorted by (table, bucket)"}
+               1: "lsh-sorted blocks", 2: "per-table units sorted by (table, bucket)",
+               3: "per-table units sorted by (bucket MinHash, table, bucket)"}
 LSH_SEED, DS_SEED, TGT_SEED = 22, 21, 23
 
 
@@ -111,7 +112,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     # N > 1: AP_SCHED_TABLE splits the (table, bucket)-sorted units (each
     # bucket read by one rank, winners MIN-reduced); the other schedules split
     # the image into block ranges (winners gathered)
-    bucket = args.schedule == 2 and world > 1
+    bucket = args.schedule in (2, 3) and world > 1
     if bucket:
         b0, b1 = 0, nb
         u0, u1 = mgpu.unit_range(cfg["L"] * nb, rank, world)
@@ -121,9 +122,12 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     tgt_host = torch.from_numpy(img).pin_memory()
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
+    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 8, "c5": 12}.get(cfg["name"], 0)
+    id_chunks = id_chunks if args.schedule in (2, 3) else 0
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0,
-                        schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0)
+                        schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0,
+                        id_chunks=id_chunks)
 
     def combine():
         if bucket:
@@ -154,7 +158,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     got = win.cpu().numpy().view(np.uint32).copy()
     # the other schedules, for comparison (cold cache, same winners)
     other_res = []
-    for other in (s for s in (0, 1, 2) if s != args.schedule and world == 1):
+    for other in (s for s in (0, 1, 2, 3) if s != args.schedule and world == 1):
         inp_o = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                               cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
                               block_count=b1 - b0, schedule=other)
@@ -235,7 +239,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         e.synchronize()
         e2e.append(s.elapsed_time(e) * 1e-3)
     cands = None
-    res = dict(cfg=cfg, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
+    res = dict(cfg=cfg, id_chunks=id_chunks, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
                units=(u0, u1), bucket=bucket,
                other=other_res,
                link=link, raw=raw, e2e=e2e, clocks=clk.summary(), t_gen=t_gen, t_pin=t_pin,
@@ -315,6 +319,7 @@ def emit_collage(args, res_all, world, METRIC):
                    "record_stride": cfg["stride"],
                    "group": args.group,
                    "schedule": SCHED_NAMES[args.schedule],
+                   "id_chunks": r0["id_chunks"],
                    "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",
                    "parallelism": (f"(table, bucket) units partitioned over {world} ranks + NCCL "
                                    "MIN reduce" if r0.get("bucket") else

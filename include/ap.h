@@ -341,11 +341,25 @@ typedef struct {
      * winners with an unsigned 64-bit MIN reduction (multi-GPU, §8(e)). */
     uint64_t unit_begin;
     uint64_t unit_count;
+    /* Record-id windows (AP_SCHED_TABLE / _MH only; 0 or 1 = off): the units
+     * run id_chunks times, pass c reading only the candidates with record
+     * id in [c*N/id_chunks, (c+1)*N/id_chunks).  A record is then needed in
+     * one pass only, whichever tables list it, so with windows whose touched
+     * records fit the cache it is filled about once (the LSH tables list it
+     * up to L times).  The keys pass keeps every block's histogram and
+     * bucket ranges in scratch (3 KiB + 8 B * L per block) for the passes.
+     * Results are identical (the per-block minimum is an atomic min). */
+    uint32_t id_chunks;
 } ap_collage_in;
 
 #define AP_SCHED_NATURAL 0
 #define AP_SCHED_LSH 1
 #define AP_SCHED_TABLE 2
+/* AP_SCHED_TABLE_MH: AP_SCHED_TABLE units sorted by (MinHash of the unit's
+ * bucket = its smallest record id, table, bucket): a bucket's units stay
+ * together and buckets of different tables sharing records come close in
+ * time.  bucket_bits <= 24.  unit_begin/unit_count slice this order. */
+#define AP_SCHED_TABLE_MH 3
 
 /* ap_collage_run — the collage kernel ("calculates the
  * histogram of each 32x32 block, computes its LSH keys, reads the candidate

@@ -16,7 +16,7 @@ AP_POLICY_CLOCK, AP_POLICY_RANDOM = 0, 1
 AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
 AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE = 0, 1, 2
-AP_SCHED_NATURAL, AP_SCHED_LSH, AP_SCHED_TABLE = 0, 1, 2
+AP_SCHED_NATURAL, AP_SCHED_LSH, AP_SCHED_TABLE, AP_SCHED_TABLE_MH = 0, 1, 2, 3
 AP_PROT_READ, AP_PROT_WRITE = 1, 2
 AP_EPERM = -9
 
@@ -49,7 +49,8 @@ class ap_collage_in(ctypes.Structure):
                 ("bucket_bits", u32), ("w", i32), ("proj_dev", vp), ("bias_dev", vp),
                 ("offsets_dev", vp), ("ids_dev", vp), ("N", u64), ("rec_stride", u32),
                 ("group", u32), ("block_begin", u64), ("block_count", u64), ("mode", i32),
-                ("raw_base", vp), ("schedule", i32), ("unit_begin", u64), ("unit_count", u64)]
+                ("raw_base", vp), ("schedule", i32), ("unit_begin", u64), ("unit_count", u64),
+                ("id_chunks", u32)]
 
 
 class ap_compute_cfg(ctypes.Structure):

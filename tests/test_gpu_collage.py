@@ -49,7 +49,7 @@ def test_index_matches_oracle(ap, K, bb):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1), (1, 2), (8, 2)])
+@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1), (1, 2), (8, 2), (1, 3), (8, 3)])
 @pytest.mark.parametrize("frames", [48, 5000])
 def test_collage_matches_oracle(ap, group, schedule, frames):
     dev = torch.device("cuda:0")
@@ -117,8 +117,9 @@ def test_collage_partitioned_blocks_equal_whole(ap):
         ap.ap_cache_destroy(cache)
 
 
+@pytest.mark.parametrize("schedule", [2, 3])
 @pytest.mark.parametrize("world", [2, 3, 8])
-def test_collage_unit_slices_min_reduce_to_whole(ap, world):
+def test_collage_unit_slices_min_reduce_to_whole(ap, world, schedule):
     """The bucket partition (mgpu.unit_range + reduce_winners_min) on one GPU:
     each slice of the (table, bucket)-sorted units runs alone into its own
     winners array; the unsigned 64-bit MIN over the slices equals the single
@@ -143,7 +144,8 @@ def test_collage_unit_slices_min_reduce_to_whole(ap, world):
             part = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
             ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
                                                       group=8, unit_begin=u0,
-                                                      unit_count=u1 - u0), part)
+                                                      unit_count=u1 - u0, schedule=schedule),
+                              part)
             f = part.view(torch.int64).view(-1) ^ flip
             acc = f if acc is None else torch.minimum(acc, f)
         got = (acc ^ flip).view(torch.int32).view(-1, 2)
@@ -159,7 +161,7 @@ def test_collage_unit_slices_min_reduce_to_whole(ap, world):
         ap.ap_cache_destroy(cache)
 
 
-@pytest.mark.parametrize("group,schedule", [(1, 1), (2, 1), (4, 1), (8, 1), (4, 2), (8, 2)])
+@pytest.mark.parametrize("group,schedule", [(1, 1), (2, 1), (4, 1), (8, 1), (4, 2), (8, 2), (8, 3)])
 @pytest.mark.parametrize("frames", [40, 3000])
 def test_unaligned_records_collage(ap, group, schedule, frames):
     """NEXT N1: 3 KiB histograms without padding, so records
@@ -186,6 +188,57 @@ def test_unaligned_records_collage(ap, group, schedule, frames):
         want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
         assert np.array_equal(win.cpu().numpy().view(np.uint32), want)
         assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("schedule,chunks,frames", [(2, 2, 40), (2, 5, 40), (3, 3, 40), (3, 7, 400)])
+def test_collage_record_id_windows(ap, schedule, chunks, frames):
+    """ap_collage_in.id_chunks: the units run once per record-id window, each
+    pass reading only candidates in its window; winners equal the one-pass
+    run and the oracle, with a cache smaller and larger than the touched
+    records, and also when the windows run over a slice of the units."""
+    dev = torch.device("cuda:0")
+    n, stride, w, bb, L, K = 2048, 4096, 2500, 8, 4, 5
+    W, H = 256, 192
+    recs, proj, bias, img, *_ = _setup(n, W, H, L, K, w, bb, seed=8)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        one = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, group=8,
+                                                  schedule=schedule), one)
+        win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_cache_reset(cache)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, group=8,
+                                                  schedule=schedule, id_chunks=chunks), win)
+        torch.cuda.synchronize()
+        assert ap.ap_last_device_error(cache) == 0
+        assert torch.equal(win, one)
+        o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+        assert np.array_equal(win.cpu().numpy().view(np.uint32), want)
+        # two unit slices, each with windows, MIN-combined
+        flip = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
+        acc = None
+        for g in range(2):
+            u0, u1 = mgpu.unit_range(L * nb, g, 2)
+            part = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+            ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                      group=8, schedule=schedule, unit_begin=u0,
+                                                      unit_count=u1 - u0, id_chunks=chunks), part)
+            f = part.view(torch.int64).view(-1) ^ flip
+            acc = f if acc is None else torch.minimum(acc, f)
+        assert torch.equal((acc ^ flip).view(torch.int32).view(-1, 2), one)
+        assert check_invariants(ap, cache, [r], frames) == []
+        from paper_conf_isca_shaharbs16_b200._lib import APError
+        with pytest.raises(APError):  # windows need per-table units
+            ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                      schedule=1, id_chunks=2), win)
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)

@@ -88,7 +88,7 @@ def test_c3_full(ap, dev):
     del f
 
 
-@pytest.mark.parametrize("schedule", [2, 1])
+@pytest.mark.parametrize("schedule", [2, 1, 3])
 def test_c4_full(ap, dev, schedule):
     """C4: 1M records (4 GiB), 1024x1024 target, L=4 K=8 2^14 buckets, 256 MiB
     cache, 8 candidates per warp: the GPU-built index and the winners of all

@@ -31,3 +31,7 @@ timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/fina
 timeout 600 python tools/fig6_sweep.py > gpurun_out/final_fig6.txt 2>&1
 timeout 300 python tools/latency.py > gpurun_out/final_latency.txt 2>&1
 echo bench-done
+timeout 300 python tools/peer_bw.py > gpurun_out/final_peer_bw.txt 2>&1
+for k in 12 16; do timeout 600 python bench.py --workload c4 --id-chunks $k --no-cpu-baseline > gpurun_out/final_c4_win$k.json 2>/dev/null; done
+timeout 900 python -m pytest tests -m gpu -q > gpurun_out/final_gpu_tests.txt 2>&1
+echo all-done
