@@ -122,7 +122,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     tgt_host = torch.from_numpy(img).pin_memory()
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
-    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 8, "c5": 12}.get(cfg["name"], 0)
+    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 12, "c5": 12}.get(cfg["name"], 0)
     id_chunks = id_chunks if args.schedule in (2, 3) else 0
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0,
@@ -338,16 +338,21 @@ def emit_collage(args, res_all, world, METRIC):
         "roofline": {"bound": "host_link", "achieved": round(fill / t0 / 1e9, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
                      "frac": round(fill / t0 / 1e9 / r0["link"], 4),
-                     "traffic": _traffic(f"k_collage<{args.group}, apointer>"),
-                     "algorithmic_bytes_per_launch": int(fill),
+                     "traffic": (lambda tr: None if tr is None else tr * max(1, r0["id_chunks"]))(
+                         _traffic(f"k_collage<{args.group}, apointer>")),
+                     "traffic_note": "DRAM bytes per step = the ncu --set full capture of one "
+                                     "k_collage launch (one record-id window pass) x the "
+                                     "step's id_chunks launches",
+                     "algorithmic_bytes_per_step": int(fill),
                      "kernel": f"k_collage<{args.group}, apointer>",
                      "peak_source": "host->device cudaMemcpy from pinned memory, this run"},
         "e2e": {"value": round(max(np.mean(r["e2e"]) for r in res_all), 6), "unit": "s",
                 "h2d_bytes_per_step": r0["h2d"], "d2h_bytes_per_step": r0["d2h"],
                 "api": "target H2D + ap_collage_run + winners D2H (cold cache)"},
-        "gpu_launches": args.steps * (3 if args.schedule else 1),
-        "gpu_launches_note": "per step: k_collage (+ k_collage_keys and k_iota32 for the LSH "
-                             "schedule; the schedule's radix sort adds cub library kernels)",
+        "gpu_launches": args.steps * ((2 + max(1, r0["id_chunks"])) if args.schedule else 1),
+        "gpu_launches_note": "per step: k_collage once per record-id window (id_chunks), plus "
+                             "k_collage_keys and k_iota32 for the sorted schedules; the "
+                             "schedule's radix sort adds cub library kernels",
         "clocks": r0["clocks"],
     }
     if r0["raw"]:

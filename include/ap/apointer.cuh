@@ -1220,6 +1220,65 @@ struct ptr {
         return reinterpret_cast<const T*>(x & XL_ADDR);
     }
 
+    /* Split-phase link -- a translation prefetch, the overlap of PAPER.md:195
+     * ("access memory in parallel with checking") applied to the minor fault:
+     * link_begin() groups the unlinked lanes by page (S5) and issues each
+     * group's optimistic PTE add (S6, relaxed: the frame data is then read
+     * with .cg loads whose addresses depend on the add's result) without
+     * waiting for it; link_finish(t) consumes it and links the lanes whose
+     * page was resident (a non-resident page's add is undone; those lanes
+     * stay unlinked and take the ordinary fault path on their next
+     * dereference).  Contract: between the two calls the warp must not enter
+     * the fault path; loads through pointers already linked, arithmetic and
+     * unlinks are fine.  Every link_begin is followed by its link_finish. */
+    struct link_ticket {
+        uint64_t old; /* leader: the PTE before the add */
+        unsigned grp; /* this lane's page group         */
+        bool need;    /* this lane took part            */
+    };
+    __device__ __forceinline__ link_ticket link_begin() {
+        const unsigned m = __activemask();
+        const bool need = !linked() && x + sizeof(T) <= r->bytes && (x % sizeof(T)) == 0;
+        const uint64_t pg = x >> lg;
+        const unsigned grp =
+            __match_any_sync(m, need ? (((unsigned long long)r->id << 48) | pg) : ~0ull);
+        uint64_t old = 0;
+        if (need && (int)detail::lane_id() == __ffs(grp) - 1) {
+            uint64_t* pte = r->pte + pg;
+            asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;"
+                         : "=l"(old) : "l"(pte), "l"((uint64_t)__popc(grp)) : "memory");
+        }
+        return link_ticket{old, grp, need};
+    }
+    __device__ __forceinline__ void link_finish(const link_ticket& t) {
+        const unsigned m = __activemask();
+        const int leader = __ffs(t.grp) - 1;
+        const bool is_leader = t.need && (int)detail::lane_id() == leader;
+        const uint64_t pg = x >> lg;
+        const bool res = (t.old >> 62) == 2;
+        if (is_leader) {
+            uint64_t* pte = r->pte + pg;
+            if (res) {
+                if (!(t.old & PTE_REF)) detail::red_or_relaxed(pte, PTE_REF);
+            } else {
+                detail::red_add_relaxed(reinterpret_cast<unsigned long long*>(pte),
+                                        (unsigned long long)(0 - (uint64_t)__popc(t.grp)));
+            }
+        }
+#ifndef AP_NO_HOT_STATS
+        const unsigned linkedm = __ballot_sync(m, is_leader && res);
+        if (linkedm && (int)detail::lane_id() == __ffs(m) - 1)
+            detail::stat_add(&(r->stats + (detail::sm_id() % STAT_SHARDS))->minor, __popc(linkedm));
+#endif
+        const uint64_t old = __shfl_sync(m, t.old, leader);
+        if (t.need && (old >> 62) == 2) {
+            const uint64_t P = 1ull << lg;
+            const uint64_t f = (old >> 32) & PTE_FRAME_MASK;
+            x = XL_VALID | ((uint64_t)(r->pool + f * P) + (x & (P - 1)));
+            page = pg;
+        }
+    }
+
     /* S4: arithmetic.  Staying inside the page keeps the link; leaving it
      * unlinks with a warp-aggregated decrement (S10). */
     __device__ __forceinline__ ptr& operator+=(int64_t d) {

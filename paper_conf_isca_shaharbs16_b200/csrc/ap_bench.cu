@@ -188,6 +188,54 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_DEREF_MINB)
     if (!a.out_copy) a.ck[t] = h;
 }
 
+/* AP_ACCESS_AHEAD: the tiled loop with a split-phase link.  The warp's next
+ * unit is linked (ptr::link_begin) right after the current unit's last tile
+ * is issued, so the PTE add travels with that tile's loads and the link
+ * (link_finish) costs no extra round trip when the warp moves on.  Units
+ * that are not whole or not a multiple of TILE deep take seq_unit. */
+template <class T>
+__device__ __forceinline__ void seq_ahead(const ap::dev_cache* c, uint32_t region,
+                                          const BenchArgs& a, uint64_t w, uint64_t lane,
+                                          uint64_t W, uint64_t nunits, uint32_t per_unit,
+                                          uint64_t& h) {
+    constexpr uint32_t E = sizeof(T);
+    if (w >= nunits) return;
+    const uint64_t per_warp = (nunits - w + W - 1) / W;
+    const uint64_t total = per_warp * a.passes;
+    const bool tiled = per_unit >= TILE && per_unit % TILE == 0;
+    ap::ptr<T> q = ap::gvmmap<T>(c, region, (w * (a.unit / E) + lane) * E);
+    uint64_t u = w;
+    for (uint64_t k = 0; k < total; ++k) {
+        const uint64_t e0 = u * (a.unit / E) + lane;
+        uint64_t un = u + W;
+        if (un >= nunits) un = w;
+        const uint64_t next_off = (un * (a.unit / E) + lane) * E;
+        if (!tiled || (u + 1) * a.unit > a.span) {
+            seq_unit<T>(q, a, e0, per_unit, (u + 1) * a.unit <= a.span, h);
+            q = ap::gvmmap<T>(c, region, next_off);
+            u = un;
+            continue;
+        }
+        uint32_t j = 0;
+        for (; j + TILE < per_unit; j += TILE) {
+            T v[TILE];
+            q.read_tile(v, 32);
+#pragma unroll
+            for (int i = 0; i < TILE; ++i) consume(a, (e0 + 32ull * (j + i)) * E, v[i], h);
+            q += 32 * TILE;
+        }
+        T v[TILE];
+        q.read_tile(v, 32);
+        ap::ptr<T> qn = ap::gvmmap<T>(c, region, next_off);
+        const auto tk = qn.link_begin();
+#pragma unroll
+        for (int i = 0; i < TILE; ++i) consume(a, (e0 + 32ull * (j + i)) * E, v[i], h);
+        q = static_cast<ap::ptr<T>&&>(qn); /* unlinks the finished unit */
+        q.link_finish(tk);
+        u = un;
+    }
+}
+
 template <class T, bool APTR>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     k_seq(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
@@ -198,6 +246,13 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
     const uint32_t per_unit = a.unit / (32 * E);
     uint64_t h = FNV_BASIS;
+    if constexpr (APTR) {
+        if (a.access == AP_ACCESS_AHEAD) {
+            seq_ahead<T>(c, region, a, w, lane, W, nunits, per_unit, h);
+            if (!a.out_copy) a.ck[t] = h;
+            return;
+        }
+    }
     for (uint32_t pass = 0; pass < a.passes; ++pass) {
         for (uint64_t u = w; u < nunits; u += W) {
             const uint64_t e0 = u * (a.unit / E) + lane;
@@ -306,7 +361,7 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
     a->page = cfg->page_bytes;
     a->span = cfg->span_bytes ? cfg->span_bytes : rg.bytes;
     a->access = cfg->access;
-    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_RANGE) return AP_EINVAL;
+    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_AHEAD) return AP_EINVAL;
     switch (cfg->pattern) {
         case AP_SEQ:
             if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;

@@ -8,8 +8,9 @@ step time is max over ranks of these per-range times, provided the host's
 memory system feeds G links at once (not measured here: one GPU per call).
 Prints, per G: per-rank seconds, fills, and max / (T1 / G).
 
-Usage: python tools/c5_partitions.py [schedule] [blocks|units]
-       (default: schedule 2 = AP_SCHED_TABLE, partitioned by units)"""
+Usage: python tools/c5_partitions.py [schedule] [blocks|units] [id_chunks]
+       (default: schedule 2 = AP_SCHED_TABLE, partitioned by units, 12 record-id
+       windows per rank as bench.py's C5 default)"""
 import os
 import sys
 
@@ -47,7 +48,8 @@ full = None
 def run_range(b0, b1, reps=2, u0=0, u1=0):
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=8, block_begin=b0, block_count=b1 - b0,
-                        schedule=sched, unit_begin=u0, unit_count=u1 - u0)
+                        schedule=sched, unit_begin=u0, unit_count=u1 - u0,
+                        id_chunks=chunks if sched in (2, 3) else 0)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     ts = []
     for _ in range(reps):
@@ -62,9 +64,10 @@ def run_range(b0, b1, reps=2, u0=0, u1=0):
     return min(ts), ap.ap_cache_stats(cache)["fill_bytes"], win
 
 
-mode = sys.argv[2] if len(sys.argv) > 2 else ("units" if sched == 2 else "blocks")
+mode = sys.argv[2] if len(sys.argv) > 2 else ("units" if sched in (2, 3) else "blocks")
+chunks = int(sys.argv[3]) if len(sys.argv) > 3 else 12
 print(f"# C5 partitions run alone on one B200 (cold 2 GiB cache each), schedule {sched}, "
-      f"partition by {mode}; {nb} blocks, {cfg['N']} records")
+      f"partition by {mode}, {chunks} record-id windows; {nb} blocks, {cfg['N']} records")
 flip = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
 t1 = None
 for G in (1, 2, 4, 8):
