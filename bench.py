@@ -514,6 +514,9 @@ def main():
     p.add_argument("--group", type=int, default=8, help="collage candidates per warp (1, 2, 4, 8)")
     p.add_argument("--schedule", type=int, default=2, help="collage: 0 = natural, 1 = LSH-sorted blocks, 2 = per-table units, 3 = per-table units in bucket-MinHash order")
     p.add_argument("--stride", type=int, default=4096, help="collage record stride (3072 = unaligned)")
+    p.add_argument("--partition", default="records", choices=["records", "units", "blocks"],
+                   help="collage, N > 1, per-table schedules: split the record ids (each GPU "
+                        "caches one shard of the file), the sorted units, or the image")
     p.add_argument("--id-chunks", type=int, default=None,
                    help="collage record-id windows (ap_collage_in.id_chunks; 0 = off; "
                         "default 12 for c4 and c5 (measured: C4 8/12/16 -> 30.3/29.2/29.1 ms, "

@@ -112,8 +112,16 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     # N > 1: AP_SCHED_TABLE splits the (table, bucket)-sorted units (each
     # bucket read by one rank, winners MIN-reduced); the other schedules split
     # the image into block ranges (winners gathered)
-    bucket = args.schedule in (2, 3) and world > 1
-    if bucket:
+    # --partition records: every rank runs all units over its slice of the
+    # record ids (each GPU caches one shard of the file), winners MIN-reduced
+    part = args.partition if args.schedule in (2, 3) else "blocks"
+    bucket = part in ("units", "records") and world > 1
+    i0, i1 = 0, 0
+    if bucket and part == "records":
+        b0, b1 = 0, nb
+        u0, u1 = 0, 0
+        i0, i1 = mgpu.id_range(cfg["N"], rank, world)
+    elif bucket:
         b0, b1 = 0, nb
         u0, u1 = mgpu.unit_range(cfg["L"] * nb, rank, world)
     else:
@@ -124,10 +132,12 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 12, "c5": 12}.get(cfg["name"], 0)
     id_chunks = id_chunks if args.schedule in (2, 3) else 0
+    if i1:  # the windows split this rank's record slice
+        id_chunks = max(1, -(-id_chunks // world))
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=args.group, block_begin=b0, block_count=b1 - b0,
                         schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0,
-                        id_chunks=id_chunks)
+                        id_chunks=id_chunks, id_begin=i0, id_end=i1)
 
     def combine():
         if bucket:
@@ -240,7 +250,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         e2e.append(s.elapsed_time(e) * 1e-3)
     cands = None
     res = dict(cfg=cfg, id_chunks=id_chunks, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
-               units=(u0, u1), bucket=bucket,
+               units=(u0, u1), bucket=bucket, records=bool(i1),
                other=other_res,
                link=link, raw=raw, e2e=e2e, clocks=clk.summary(), t_gen=t_gen, t_pin=t_pin,
                t_index=t_index, h2d=int(tgt_host.numel()), d2h=int(win.numel() * 4),
@@ -266,7 +276,8 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
                                   threads=os.cpu_count() or 1)
             ok = ok and bool(np.array_equal(want, fw[rb0:rb0 + k]))
         res["gathered_parity"] = dict(ranks=world, blocks_per_rank=16, equal=ok,
-                                      partition="buckets (units)" if bucket else "blocks")
+                                      partition=("records (id slices)" if i1 else "buckets (units)")
+                                      if bucket else "blocks")
     if rank == 0 and not args.no_cpu_baseline:
         import oracle
         o_off = off.cpu().numpy().view(np.uint32)
@@ -321,7 +332,9 @@ def emit_collage(args, res_all, world, METRIC):
                    "schedule": SCHED_NAMES[args.schedule],
                    "id_chunks": r0["id_chunks"],
                    "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",
-                   "parallelism": (f"(table, bucket) units partitioned over {world} ranks + NCCL "
+                   "parallelism": ((f"record-id slices (file shards) over {world} ranks, all units "
+                                    "each + NCCL MIN reduce") if r0.get("records") else
+                                   f"(table, bucket) units partitioned over {world} ranks + NCCL "
                                    "MIN reduce" if r0.get("bucket") else
                                    f"blocks partitioned over {world} rank(s) + NCCL gather")},
         "collage": {"blocks_rank0": r0["b1"] - r0["b0"],

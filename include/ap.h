@@ -351,6 +351,14 @@ typedef struct {
      * bucket ranges in scratch (3 KiB + 8 B * L per block) for the passes.
      * Results are identical (the per-block minimum is an atomic min). */
     uint32_t id_chunks;
+    /* Record-id range (per-table schedules only; id_end 0 = all records):
+     * only candidates with id in [id_begin, id_end) are read; id_chunks then
+     * splits this range.  Multi-GPU "by records": rank r takes the r-th
+     * slice of the ids and runs every unit, so each GPU's page cache only
+     * ever holds its own shard of the file; the partial winners are combined
+     * with the same 64-bit MIN reduction as the bucket partition. */
+    uint32_t id_begin;
+    uint32_t id_end;
 } ap_collage_in;
 
 #define AP_SCHED_NATURAL 0

@@ -230,7 +230,7 @@ def ap_bench_latency(cache, region, op, reps=1000):
 def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev, ids_dev, N,
                rec_stride=4096, group=1, block_begin=0, block_count=None,
                mode=AP_MODE_APOINTER, raw_base=None, L=None, K=None, schedule=AP_SCHED_TABLE,
-               unit_begin=0, unit_count=0, id_chunks=0):
+               unit_begin=0, unit_count=0, id_chunks=0, id_begin=0, id_end=0):
     L = proj_dev.shape[0] if L is None else L
     K = proj_dev.shape[1] if K is None else K
     nb = (W // 32) * (H // 32)
@@ -238,7 +238,7 @@ def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev
     return ap_collage_in(_ptr(target_dev), W, H, L, K, bucket_bits, w, _ptr(proj_dev),
                          _ptr(bias_dev), _ptr(offsets_dev), _ptr(ids_dev), N, rec_stride, group,
                          block_begin, block_count, mode, _ptr(raw_base), schedule, unit_begin,
-                         unit_count, id_chunks)
+                         unit_count, id_chunks, id_begin, id_end)
 
 
 def ap_collage_run(cache, region, inp, winners_dev, stream=None):

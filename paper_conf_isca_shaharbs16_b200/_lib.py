@@ -50,7 +50,7 @@ class ap_collage_in(ctypes.Structure):
                 ("offsets_dev", vp), ("ids_dev", vp), ("N", u64), ("rec_stride", u32),
                 ("group", u32), ("block_begin", u64), ("block_count", u64), ("mode", i32),
                 ("raw_base", vp), ("schedule", i32), ("unit_begin", u64), ("unit_count", u64),
-                ("id_chunks", u32)]
+                ("id_chunks", u32), ("id_begin", u32), ("id_end", u32)]
 
 
 class ap_compute_cfg(ctypes.Structure):

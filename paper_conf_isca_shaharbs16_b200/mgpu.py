@@ -9,6 +9,12 @@
   several ranks, so the winners are combined with one MIN reduction of the
   64-bit (dist << 32 | idx) words (R-A3's lexicographic order).
 
+* by records (AP_SCHED_TABLE with ap_collage_in.id_begin/id_end): rank r
+  runs every unit but reads only candidates whose record id lies in its
+  contiguous slice of the file, so each GPU's page cache holds one shard of
+  the file and every record is filled by exactly one rank (a data-parallel
+  split of the file itself); winners are MIN-reduced like the bucket split.
+
 NCCL over NVLink on GPUs; gloo in the CPU tests.  Marshalling only.
 """
 
@@ -44,6 +50,11 @@ def gather_winners(win, rank, world, dist, nblocks, dst=0):
 def unit_range(nunits, rank, world):
     """Contiguous range [u0, u1) of the sorted units for rank `rank`."""
     return rank * nunits // world, (rank + 1) * nunits // world
+
+
+def id_range(nrecords, rank, world):
+    """Contiguous record-id slice [i0, i1) of rank `rank` (by-records split)."""
+    return rank * nrecords // world, (rank + 1) * nrecords // world
 
 
 def reduce_winners_min(win, rank, world, dist, dst=0):

@@ -242,3 +242,55 @@ def test_collage_record_id_windows(ap, schedule, chunks, frames):
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("world,chunks", [(2, 0), (3, 2), (8, 1)])
+def test_collage_record_slices_min_reduce_to_whole(ap, world, chunks):
+    """The by-records partition (mgpu.id_range + reduce_winners_min) on one
+    GPU: each rank's record-id slice, all units, runs alone; the MIN over
+    the slices equals the single run and the oracle; each slice fills only
+    pages of its own records."""
+    dev = torch.device("cuda:0")
+    n, stride, w, bb, L, K = 2048, 4096, 2500, 8, 4, 5
+    W, H = 256, 192
+    recs, proj, bias, img, *_ = _setup(n, W, H, L, K, w, bb, seed=9)
+    cache = ap.ap_cache_create(60, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        full = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                  group=8), full)
+        flip = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
+        acc = None
+        for g in range(world):
+            i0, i1 = mgpu.id_range(n, g, world)
+            ap.ap_cache_reset(cache)
+            part = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+            ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                      group=8, id_chunks=chunks, id_begin=i0,
+                                                      id_end=i1), part)
+            torch.cuda.synchronize()
+            # only this slice's record pages were ever filled
+            pte = ap.ap_region_dump_pte(cache, r)
+            touched = np.nonzero((pte >> np.uint64(62)) != 0)[0]
+            assert touched.size == 0 or (touched.min() >= i0 and touched.max() < i1)
+            f = part.view(torch.int64).view(-1) ^ flip
+            acc = f if acc is None else torch.minimum(acc, f)
+        got = (acc ^ flip).view(torch.int32).view(-1, 2)
+        assert ap.ap_last_device_error(cache) == 0
+        assert torch.equal(got, full)
+        o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+        assert np.array_equal(got.cpu().numpy().view(np.uint32), want)
+        from paper_conf_isca_shaharbs16_b200._lib import APError
+        for bad in (dict(id_begin=5, id_end=5), dict(id_begin=0, id_end=n + 1),
+                    dict(id_begin=1, id_end=9, schedule=1)):
+            with pytest.raises(APError):
+                ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
+                                                          **bad), part)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)

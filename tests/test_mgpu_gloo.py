@@ -119,3 +119,60 @@ def test_unit_ranges_cover_exactly():
             rs = [mgpu.unit_range(nu, r, world) for r in range(world)]
             assert rs[0][0] == 0 and rs[-1][1] == nu
             assert all(rs[i][1] == rs[i + 1][0] for i in range(world - 1))
+
+
+def _restrict_index(off, ids, i0, i1):
+    """The bucket CSR with every id outside [i0, i1) dropped (test-side
+    marshalling of the by-records split; the oracle itself is unchanged)."""
+    off_r, ids_r = np.zeros_like(off), np.zeros_like(ids)
+    for t in range(off.shape[0]):
+        k = 0
+        for b in range(off.shape[1] - 1):
+            off_r[t, b] = k
+            seg = ids[t, off[t, b]:off[t, b + 1]]
+            seg = seg[(seg >= i0) & (seg < i1)]
+            ids_r[t, k:k + seg.size] = seg
+            k += seg.size
+        off_r[t, -1] = k
+    return off_r, ids_r
+
+
+def _worker_records(rank, world, port, q):
+    """By-records partition: rank r sees only candidates whose record id is
+    in mgpu.id_range(N, r, world); the MIN reduction gives the whole answer."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, stride, w, bb, recs, proj, bias, img, off, ids = _setup()
+    i0, i1 = mgpu.id_range(n, rank, world)
+    off_r, ids_r = _restrict_index(off, ids, i0, i1)
+    part = oracle.collage(img, proj, bias, w, bb, recs, stride, n, off_r, ids_r, threads=1)
+    full = mgpu.reduce_winners_min(torch.from_numpy(part.view(np.int32).copy()), rank, world, dist)
+    if rank == 0:
+        q.put(full.numpy().view(np.uint32).copy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_record_partition_min_reduces_to_the_whole_answer(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_records, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    n, stride, w, bb, recs, proj, bias, img, off, ids = _setup()
+    want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, off, ids, threads=1)
+    assert np.array_equal(got, want)
+
+
+def test_id_ranges_cover_exactly():
+    for n in (1, 9, 1500, 10_000_000):
+        for world in (1, 2, 3, 8):
+            rs = [mgpu.id_range(n, r, world) for r in range(world)]
+            assert rs[0][0] == 0 and rs[-1][1] == n
+            assert all(rs[i][1] == rs[i + 1][0] for i in range(world - 1))

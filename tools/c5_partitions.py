@@ -8,7 +8,7 @@ step time is max over ranks of these per-range times, provided the host's
 memory system feeds G links at once (not measured here: one GPU per call).
 Prints, per G: per-rank seconds, fills, and max / (T1 / G).
 
-Usage: python tools/c5_partitions.py [schedule] [blocks|units] [id_chunks]
+Usage: python tools/c5_partitions.py [schedule] [blocks|units|records] [id_chunks]
        (default: schedule 2 = AP_SCHED_TABLE, partitioned by units, 12 record-id
        windows per rank as bench.py's C5 default)"""
 import os
@@ -45,11 +45,12 @@ nb = (cfg["W"] // 32) * (cfg["H"] // 32)
 full = None
 
 
-def run_range(b0, b1, reps=2, u0=0, u1=0):
+def run_range(b0, b1, reps=2, u0=0, u1=0, i0=0, i1=0, nwin=None):
     inp = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids, cfg["N"],
                         cfg["stride"], group=8, block_begin=b0, block_count=b1 - b0,
                         schedule=sched, unit_begin=u0, unit_count=u1 - u0,
-                        id_chunks=chunks if sched in (2, 3) else 0)
+                        id_chunks=(chunks if nwin is None else nwin) if sched in (2, 3) else 0,
+                        id_begin=i0, id_end=i1)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
     ts = []
     for _ in range(reps):
@@ -76,13 +77,16 @@ for G in (1, 2, 4, 8):
         if mode == "units":  # rank r: a slice of the (table, bucket)-sorted units, all blocks
             u0, u1 = mgpu.unit_range(cfg["L"] * nb, r, G)
             t, fb, w = run_range(0, nb, u0=u0, u1=u1)
+        elif mode == "records":  # rank r: all units, records [i0, i1) only
+            i0, i1 = mgpu.id_range(cfg["N"], r, G)
+            t, fb, w = run_range(0, nb, i0=i0, i1=i1, nwin=max(1, -(-chunks // G)))
         else:
             b0, b1 = mgpu.block_range(nb, r, G)
             t, fb, w = run_range(b0, b1)
         per.append(t)
         fills.append(fb)
         parts.append(w)
-    if mode == "units":  # the MIN reduction of reduce_winners_min, on one device
+    if mode in ("units", "records"):  # the MIN reduction of reduce_winners_min, on one device
         acc = parts[0].view(torch.int64).view(-1) ^ flip
         for w in parts[1:]:
             acc = torch.minimum(acc, w.view(torch.int64).view(-1) ^ flip)
