@@ -236,6 +236,44 @@ __device__ __forceinline__ void seq_ahead(const ap::dev_cache* c, uint32_t regio
     }
 }
 
+/* AP_ACCESS_PAIR: the tiled loop over two units at a time.  Both units'
+ * pointers are linked together (two split-phase links: both PTE adds are in
+ * flight at once, one round trip for two links), then the units are read
+ * one after the other with the plain tile loop. */
+template <class T>
+__device__ __forceinline__ void seq_pair(const ap::dev_cache* c, uint32_t region,
+                                         const BenchArgs& a, uint64_t w, uint64_t lane,
+                                         uint64_t W, uint64_t nunits, uint32_t per_unit,
+                                         uint64_t& h) {
+    constexpr uint32_t E = sizeof(T);
+    for (uint32_t pass = 0; pass < a.passes; ++pass) {
+        for (uint64_t u = w; u < nunits; u += 2 * W) {
+            const uint64_t u1 = u + W;
+            const bool two = u1 < nunits && (u1 + 1) * a.unit <= a.span && (u + 1) * a.unit <= a.span;
+            ap::ptr<T> q0 = ap::gvmmap<T>(c, region, (u * (a.unit / E) + lane) * E);
+            if (!two) {
+                seq_unit<T>(q0, a, u * (a.unit / E) + lane, per_unit, (u + 1) * a.unit <= a.span, h);
+                if (u1 < nunits) {
+                    ap::ptr<T> q1 = ap::gvmmap<T>(c, region, (u1 * (a.unit / E) + lane) * E);
+                    seq_unit<T>(q1, a, u1 * (a.unit / E) + lane, per_unit,
+                                (u1 + 1) * a.unit <= a.span, h);
+                }
+                continue;
+            }
+            ap::ptr<T> q1 = ap::gvmmap<T>(c, region, (u1 * (a.unit / E) + lane) * E);
+            {
+                const auto t0 = q0.link_begin();
+                const auto t1 = q1.link_begin();
+                q0.link_finish(t0);
+                q1.link_finish(t1);
+            }
+            seq_unit<T>(q0, a, u * (a.unit / E) + lane, per_unit, true, h);
+            q0.release();
+            seq_unit<T>(q1, a, u1 * (a.unit / E) + lane, per_unit, true, h);
+        }
+    }
+}
+
 template <class T, bool APTR>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     k_seq(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
@@ -246,13 +284,6 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
     const uint32_t per_unit = a.unit / (32 * E);
     uint64_t h = FNV_BASIS;
-    if constexpr (APTR) {
-        if (a.access == AP_ACCESS_AHEAD) {
-            seq_ahead<T>(c, region, a, w, lane, W, nunits, per_unit, h);
-            if (!a.out_copy) a.ck[t] = h;
-            return;
-        }
-    }
     for (uint32_t pass = 0; pass < a.passes; ++pass) {
         for (uint64_t u = w; u < nunits; u += W) {
             const uint64_t e0 = u * (a.unit / E) + lane;
@@ -279,6 +310,24 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
             }
         }
     }
+    if (!a.out_copy) a.ck[t] = h;
+}
+
+/* The split-phase link experiments (AP_ACCESS_AHEAD, AP_ACCESS_PAIR) get a
+ * kernel of their own, so adding them does not perturb ptxas's allocation of
+ * k_seq's tile loop (tests/test_sass.py). */
+template <class T>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
+    k_seq_split(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t w = t >> 5, lane = t & 31;
+    const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
+    const uint32_t per_unit = a.unit / (32 * E);
+    uint64_t h = FNV_BASIS;
+    if (a.access == AP_ACCESS_AHEAD) seq_ahead<T>(c, region, a, w, lane, W, nunits, per_unit, h);
+    else seq_pair<T>(c, region, a, w, lane, W, nunits, per_unit, h);
     if (!a.out_copy) a.ck[t] = h;
 }
 
@@ -318,6 +367,8 @@ cudaError_t launch_t(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg
         case AP_SEQ:
             if (cfg->access == AP_ACCESS_DEREF)
                 k_seq_deref<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            else if (APTR && (cfg->access == AP_ACCESS_AHEAD || cfg->access == AP_ACCESS_PAIR))
+                k_seq_split<T><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             else
                 k_seq<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             break;
@@ -361,7 +412,7 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
     a->page = cfg->page_bytes;
     a->span = cfg->span_bytes ? cfg->span_bytes : rg.bytes;
     a->access = cfg->access;
-    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_AHEAD) return AP_EINVAL;
+    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_PAIR) return AP_EINVAL;
     switch (cfg->pattern) {
         case AP_SEQ:
             if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;

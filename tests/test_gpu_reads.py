@@ -27,7 +27,7 @@ def _run(ap, cache, region, cfg, nthreads, dev, out_bytes=None):
     return out.cpu().numpy()
 
 
-ACCESS = [0, 2, 3]  # AP_ACCESS_TILE, AP_ACCESS_RANGE, AP_ACCESS_AHEAD
+ACCESS = [0, 2, 3, 4]  # AP_ACCESS_TILE, _RANGE, _AHEAD, _PAIR
 
 
 @pytest.mark.parametrize("access", ACCESS)

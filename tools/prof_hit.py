@@ -51,7 +51,7 @@ def t(fn, n=5):
 
 tr = t(lambda: ap.ap_bench_read(cache, r, cfg_raw, out2))
 nb = span * passes
-for acc, name in ((ap.AP_ACCESS_TILE, "tile"), (ap.AP_ACCESS_AHEAD, "ahead"), (ap.AP_ACCESS_RANGE, "range"), (ap.AP_ACCESS_DEREF, "deref")):
+for acc, name in ((ap.AP_ACCESS_TILE, "tile"), (ap.AP_ACCESS_AHEAD, "ahead"), (ap.AP_ACCESS_PAIR, "pair"), (ap.AP_ACCESS_RANGE, "range"), (ap.AP_ACCESS_DEREF, "deref")):
     cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=passes, span_bytes=span,
                        access=acc)
     ta = t(lambda: ap.ap_bench_read(cache, r, cfg, out))
