@@ -122,5 +122,58 @@ ap.ap_munmap(c, r2)
 ap.ap_munmap(c, r1)
 check("copy reaches the file", np.array_equal(dst, src))
 ap.ap_cache_destroy(c)
+# per-table schedules with record-id windows and a record-id range (the
+# by-records multi-GPU share), over a 12-frame cache
+c = ap.ap_cache_create(12, 4096)
+r = ap.ap_mmap(c, recs)
+for sch in (2, 3):
+    for kw in (dict(id_chunks=3), dict(id_chunks=2, id_begin=0, id_end=n // 2)):
+        win = torch.zeros((8, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(c, r, ap.collage_in(tgt, 128, 64, pd, bd, w, bb, off, ids, n, group=8,
+                                              schedule=sch, **kw), win)
+        torch.cuda.synchronize()
+        if "id_end" in kw:
+            win2 = torch.zeros((8, 2), dtype=torch.int32, device=dev)
+            ap.ap_collage_run(c, r, ap.collage_in(tgt, 128, 64, pd, bd, w, bb, off, ids, n,
+                                                  group=8, schedule=sch, id_begin=n // 2), win2)
+            torch.cuda.synchronize()
+            f = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
+            win = ((torch.minimum(win.view(torch.int64).view(-1) ^ f,
+                                  win2.view(torch.int64).view(-1) ^ f)) ^ f).view(torch.int32).view(-1, 2)
+        check(f"collage schedule={sch} {sorted(kw)}", np.array_equal(win.cpu().numpy().view(np.uint32), want))
+check("windows invariants", check_invariants(ap, c, [r], 12) == [])
+check("windows device error", ap.ap_last_device_error(c) == 0)
+ap.ap_munmap(c, r)
+ap.ap_cache_destroy(c)
+
+# peer caches: two 3-frame caches that are each other's peer, reading at once
+fp = make_file(32 * 4096, 4)
+ca, cb = ap.ap_cache_create(3, 4096), ap.ap_cache_create(3, 4096)
+ra, rb = ap.ap_mmap(ca, fp), ap.ap_mmap(cb, fp)
+ap.ap_region_add_peer(ca, ra, cb, rb)
+ap.ap_region_add_peer(cb, rb, ca, ra)
+sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+cka = torch.zeros(128, dtype=torch.int64, device=dev)
+ckb = torch.zeros(128, dtype=torch.int64, device=dev)
+ap.ap_bench_read(ca, ra, ap.bench_cfg(ap.AP_UNIFORM, 4, 1, 128, reads_per_thread=4, seed=7), cka, sa)
+ap.ap_bench_read(cb, rb, ap.bench_cfg(ap.AP_UNIFORM, 4, 1, 128, reads_per_thread=4, seed=8), ckb, sb)
+torch.cuda.synchronize()
+check("peers a", np.array_equal(cka.cpu().numpy().view(np.uint64), oracle.read_uniform(fp, fp.nbytes, 4, 128, 4, 7)))
+check("peers b", np.array_equal(ckb.cpu().numpy().view(np.uint64), oracle.read_uniform(fp, fp.nbytes, 4, 128, 4, 8)))
+check("peers invariants", check_invariants(ap, ca, [ra], 3) == [] and check_invariants(ap, cb, [rb], 3) == [])
+# split-phase link styles
+for acc in (ap.AP_ACCESS_AHEAD, ap.AP_ACCESS_PAIR):
+    ck2 = torch.zeros(128, dtype=torch.int64, device=dev)
+    ap.ap_bench_read(ca, ra, ap.bench_cfg(ap.AP_SEQ, 16, 1, 128, unit_bytes=4096, access=acc), ck2)
+    torch.cuda.synchronize()
+    check(f"seq access={acc} (peers on)", np.array_equal(
+        ck2.cpu().numpy().view(np.uint64), oracle.read_seq(fp, fp.nbytes, 4096, 16, 128, 1)))
+check("peers device error", ap.ap_last_device_error(ca) == 0 and ap.ap_last_device_error(cb) == 0)
+ap.ap_region_clear_peers(ca, ra)
+ap.ap_region_clear_peers(cb, rb)
+ap.ap_munmap(ca, ra)
+ap.ap_munmap(cb, rb)
+ap.ap_cache_destroy(ca)
+ap.ap_cache_destroy(cb)
 print("ALL OK" if ok else "FAILURES")
 sys.exit(0 if ok else 1)
