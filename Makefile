@@ -1,6 +1,7 @@
 # Builds the three native libraries in-tree (the .so files travel to the GPU
 # box with the gpurun snapshot; they are git-ignored).
 #   paper_conf_isca_shaharbs16_b200/libapointer.so  -- the product (CUDA, sm_100a)
+#   paper_conf_isca_shaharbs16_b200/libapointer_hash.so -- N4 ablation: hash-table page table
 #   oracle/liboracle.so                             -- CPU oracle (test infrastructure)
 #   synth/libsynth.so                               -- seeded input generators
 NVCC    ?= /usr/local/cuda/bin/nvcc
@@ -15,7 +16,7 @@ CFLAGS  := -O2 -fopenmp -fPIC -Wall -Wextra -std=c11
 CU_SRCS := $(wildcard $(CSRC)/*.cu)
 CU_HDRS := $(wildcard $(CSRC)/*.cuh) $(wildcard include/*.h) $(wildcard include/ap/*.cuh)
 
-all: synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so
+all: synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so $(PKG)/libapointer_hash.so
 
 synth/libsynth.so: synth/synth.c
 	$(HOSTCC) $(CFLAGS) -shared $< -o $@ -lm
@@ -26,12 +27,16 @@ oracle/liboracle.so: oracle/oracle.c
 $(PKG)/libapointer.so: $(CU_SRCS) $(CU_HDRS)
 	$(NVCC) $(NVFLAGS) -shared $(CU_SRCS) -o $@ -lcuda
 
+# N4 ablation: the paper's hash-table page table instead of the dense PTE array
+$(PKG)/libapointer_hash.so: $(CU_SRCS) $(CU_HDRS)
+	$(NVCC) $(NVFLAGS) -DAP_PT_HASH -shared $(CU_SRCS) -o $@ -lcuda
+
 host: synth/libsynth.so oracle/liboracle.so
 
 sass: $(PKG)/libapointer.so
 	/usr/local/cuda/bin/cuobjdump -sass $< > build_sass.txt
 
 clean:
-	rm -f synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so
+	rm -f synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so $(PKG)/libapointer_hash.so
 
 .PHONY: all host clean sass

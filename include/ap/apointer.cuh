@@ -313,6 +313,41 @@ __device__ __forceinline__ uint64_t sm64(uint64_t x) {
     return z ^ (z >> 31);
 }
 
+/* -------------------------------------------------------------------------
+ * N4 ablation (-DAP_PT_HASH): the paper's page table -- one concurrent hash
+ * table indexing the pages of all files, 16x the number of frames, lock-free
+ * reads -- instead of the dense per-region PTE array.  A slot
+ * is {key = (region + 1) << 48 | page, the same 64-bit PTE}; linear probing
+ * from splitmix64(key).  In this build the region descriptor's `pte` points
+ * at the cache's slot table and `pad_` holds log2(slots).  A key, once
+ * inserted, keeps its slot while the region is mapped (no removal, so no
+ * probe chain ever breaks and a slot never changes pages); ap_mmap sizes the
+ * table to at least twice the pages mapped.  Dense builds never compile
+ * this. */
+#ifdef AP_PT_HASH
+constexpr uint64_t PT_TOMB = ~0ull;
+__device__ __forceinline__ uint64_t* pt_find(const dev_region* r, uint64_t pg, bool insert) {
+    uint64_t* slots = r->pte;
+    const uint64_t mask = (1ull << r->pad_) - 1;
+    const uint64_t key = ((uint64_t)(r->id + 1) << 48) | pg;
+    uint64_t h = sm64(key) & mask;
+    for (uint64_t i = 0; i <= mask; ++i, h = (h + 1) & mask) {
+        uint64_t k = ld_relaxed(slots + 2 * h);
+        if (k == 0 && insert) {
+            k = atomicCAS(reinterpret_cast<unsigned long long*>(slots + 2 * h), 0ull,
+                          (unsigned long long)key);
+            if (k == 0) return slots + 2 * h + 1;
+        }
+        if (k == key) return slots + 2 * h + 1;
+        if (k == 0) return nullptr;
+    }
+    return nullptr;
+}
+#define AP_PTE_AT(r, pg) ::ap::detail::pt_find((r), (pg), false)
+#else
+#define AP_PTE_AT(r, pg) ((r)->pte + (pg))
+#endif
+
 /* Frame-data loads bypass L1 (.cg): a recycled frame can never be served
  * from a stale L1 line, and the data is streamed once anyway. */
 template <class T> __device__ __forceinline__ T ld_data(const T* p);
@@ -375,7 +410,7 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
 #ifdef AP_DEBUG
         printf("[unlink] w%u m%08x grp%08x n%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, grp, n, (unsigned long long)page);
 #endif
-        red_unlink(r->pte + page, (uint64_t)0 - (uint64_t)n);
+        red_unlink(AP_PTE_AT(r, page), (uint64_t)0 - (uint64_t)n);
 #if defined(AP_COUNT_UNLINKS) && !defined(AP_NO_HOT_STATS)
         /* opt-in: one more atomic per unlink cost a third of the minor-fault
          * throughput (M2r 14.5 -> 10.0 G reads/s), so it is off by default */
@@ -465,8 +500,13 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         const uint64_t own = ld_relaxed(c->owner + f);
         if (own) {
             const dev_region* vr = c->regions + ((own >> 48) - 1);
-            q = vr->pte + (own & PAGE_MASK48);
+            q = AP_PTE_AT(vr, own & PAGE_MASK48);
+#ifdef AP_PT_HASH
+            /* the owner entry can become visible before the key's insert */
+            e = q ? ld_relaxed(q) : 0;
+#else
             e = ld_relaxed(q);
+#endif
             if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f && (e & PTE_RC_MASK) == 0) {
                 if (c->policy == POLICY_CLOCK && (e & PTE_REF)) cas_relaxed(q, e, e & ~PTE_REF);
                 else elig = true;
@@ -510,7 +550,8 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
 #ifdef AP_DEBUG
     if (still && (int)lane == first) {
         const uint64_t own0 = ld_relaxed(c->owner);
-        const uint64_t e0 = own0 ? ld_relaxed(c->regions[(own0 >> 48) - 1].pte + (own0 & PAGE_MASK48)) : 0;
+        const uint64_t* q0 = own0 ? AP_PTE_AT(&c->regions[(own0 >> 48) - 1], own0 & PAGE_MASK48) : nullptr;
+        const uint64_t e0 = q0 ? ld_relaxed(q0) : 0;
         if ((clock64() & 0xfffff) < 200)
             printf("[nofree] sm %u warp %u m %08x own0 %llx e0 %llx hand %llu\n", sm_id(),
                    (unsigned)(threadIdx.x >> 5), m, (unsigned long long)own0, (unsigned long long)e0,
@@ -642,7 +683,11 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         const int leader = __ffs(grp) - 1;
         const bool is_leader = need && (int)lane == leader;
         const uint32_t n = __popc(grp);
+#ifdef AP_PT_HASH
+        uint64_t* pte = is_leader ? pt_find(r, pg, true) : nullptr;
+#else
         uint64_t* pte = r->pte + pg;
+#endif
 
         /* Phase A (leaders, lane-parallel; R-A13): minor faults link at once;
          * up to max_claims leaders (lane order) may claim an EMPTY entry. */
@@ -819,13 +864,20 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
     const bool is_leader = need && (int)lane_id() == leader;
     uint64_t old = 0;
     if (is_leader) {
+#ifdef AP_PT_HASH
+        uint64_t* pte = pt_find(r, pg, false); /* no slot: not resident */
+        if (pte) {
+#else
         uint64_t* pte = r->pte + pg;
-        old = add_link(pte, __popc(grp));
-        if ((old >> 62) == 2) {
-            if (!(old & PTE_REF)) red_or_relaxed(pte, PTE_REF);
-        } else {
-            red_add_relaxed(reinterpret_cast<unsigned long long*>(pte),
-                            (unsigned long long)(0 - (uint64_t)__popc(grp)));
+        {
+#endif
+            old = add_link(pte, __popc(grp));
+            if ((old >> 62) == 2) {
+                if (!(old & PTE_REF)) red_or_relaxed(pte, PTE_REF);
+            } else {
+                red_add_relaxed(reinterpret_cast<unsigned long long*>(pte),
+                                (unsigned long long)(0 - (uint64_t)__popc(grp)));
+            }
         }
     }
 #ifndef AP_NO_HOT_STATS /* ablation: no counters on the inline link / unlink */
@@ -961,7 +1013,7 @@ __device__ AP_SLOW_ATTR slow_out<T> store_slow(unsigned m, uint64_t x, uint64_t 
         const bool mark = lnk && !(x & XL_DIRTY);
         const unsigned long long key = mark ? (((unsigned long long)r->id << 48) | page) : ~0ull;
         const unsigned grp = __match_any_sync(m, key);
-        if (mark && (int)lane == __ffs(grp) - 1) red_or_relaxed(r->pte + page, PTE_DIRTY);
+        if (mark && (int)lane == __ffs(grp) - 1) red_or_relaxed(AP_PTE_AT(r, page), PTE_DIRTY);
         if (lnk) {
             x |= XL_DIRTY;
             st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
@@ -992,7 +1044,7 @@ __device__ AP_SLOW_ATTR slow_out<T> store_slow(unsigned m, uint64_t x, uint64_t 
             page = o.page;
             const bool ok = (x >> 63) != 0;
             const unsigned okm = __ballot_sync(mg, ok);
-            if (ok && (int)lane == __ffs(okm) - 1) red_or_relaxed(r->pte + page, PTE_DIRTY);
+            if (ok && (int)lane == __ffs(okm) - 1) red_or_relaxed(AP_PTE_AT(r, page), PTE_DIRTY);
             if (ok) {
                 x |= XL_DIRTY;
                 st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
@@ -1244,7 +1296,11 @@ struct ptr {
             __match_any_sync(m, need ? (((unsigned long long)r->id << 48) | pg) : ~0ull);
         uint64_t old = 0;
         if (need && (int)detail::lane_id() == __ffs(grp) - 1) {
-            uint64_t* pte = r->pte + pg;
+            uint64_t* pte = AP_PTE_AT(r, pg);
+#ifdef AP_PT_HASH
+            if (!pte) old = 3ull << 62; /* no slot: nothing added (no early return: */
+            else                        /* the warp must stay converged)            */
+#endif
             asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;"
                          : "=l"(old) : "l"(pte), "l"((uint64_t)__popc(grp)) : "memory");
         }
@@ -1256,8 +1312,8 @@ struct ptr {
         const bool is_leader = t.need && (int)detail::lane_id() == leader;
         const uint64_t pg = x >> lg;
         const bool res = (t.old >> 62) == 2;
-        if (is_leader) {
-            uint64_t* pte = r->pte + pg;
+        if (is_leader && (t.old >> 62) != 3) {
+            uint64_t* pte = AP_PTE_AT(r, pg);
             if (res) {
                 if (!(t.old & PTE_REF)) detail::red_or_relaxed(pte, PTE_REF);
             } else {

@@ -44,6 +44,9 @@ struct ap_cache_s {
     ap::dev_cache h{};                /* host mirror         */
     std::vector<ap_region_host> reg;
     int num_sms = 148;
+    uint64_t* slots = nullptr; /* -DAP_PT_HASH: the hash page table (N4 ablation) */
+    uint32_t slot_bits = 0;
+    uint64_t slot_keys = 0;    /* keys inserted at most (mapped pages + tombstones) */
     void* scratch = nullptr; /* grown on demand (collage schedule) */
     size_t scratch_bytes = 0;
 };

@@ -36,7 +36,12 @@ extern "C" const char* ap_strerror(int code) {
 }
 
 extern "C" const char* ap_version(void) {
-    return "apointer-b200 0.1 (sm_100a; long apointer, no TLB, clock eviction)";
+#ifdef AP_PT_HASH
+    return "apointer-b200 0.1 (sm_100a; long apointer, no TLB, clock eviction; "
+           "hash-table page table)";
+#else
+    return "apointer-b200 0.1 (sm_100a; long apointer, no TLB, clock eviction; dense page table)";
+#endif
 }
 
 void* ap_scratch(ap_cache_s* c, size_t bytes) {
@@ -81,6 +86,38 @@ __global__ void k_scan_pte(const uint64_t* pte, uint64_t n, int* flag) {
     if (f) atomicOr(flag, f);
 }
 
+#ifdef AP_PT_HASH
+/* hash page table (N4 ablation): per-slot scans of one region's keys */
+__global__ void k_scan_slots(const uint64_t* slots, uint64_t n, uint64_t tag, int* flag) {
+    int f = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        if ((slots[2 * i] >> 48) != tag || slots[2 * i] == ap::detail::PT_TOMB) continue;
+        const uint64_t e = slots[2 * i + 1];
+        if (e & ap::PTE_RC_MASK) f |= 1;
+        if ((e >> 62) == 1) f |= 2;
+    }
+    if (f) atomicOr(flag, f);
+}
+__global__ void k_tomb_slots(uint64_t* slots, uint64_t n, uint64_t tag) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        if ((slots[2 * i] >> 48) == tag && slots[2 * i] != ap::detail::PT_TOMB) {
+            slots[2 * i] = ap::detail::PT_TOMB;
+            slots[2 * i + 1] = 0;
+        }
+}
+__global__ void k_dump_slots(const uint64_t* slots, uint64_t n, uint64_t tag, uint64_t* dense,
+                             uint64_t npages) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t k = slots[2 * i];
+        if ((k >> 48) == tag && k != ap::detail::PT_TOMB && (k & ap::PAGE_MASK48) < npages)
+            dense[k & ap::PAGE_MASK48] = slots[2 * i + 1];
+    }
+}
+#endif
+
 __global__ void k_drop_owner(uint64_t* owner, uint64_t frames, uint64_t tag) {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < frames;
          i += (uint64_t)gridDim.x * blockDim.x)
@@ -108,12 +145,16 @@ __global__ void k_writeback(const ap::dev_cache* __restrict__ c, uint32_t region
     const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) / 32;
     const uint64_t nwarps = (uint64_t)gridDim.x * blockDim.x / 32;
     for (uint64_t p = warp; p < r->npages; p += nwarps) {
-        const uint64_t e = r->pte[p];
+        uint64_t* q = AP_PTE_AT(r, p);
+#ifdef AP_PT_HASH
+        if (!q) continue;
+#endif
+        const uint64_t e = *q;
         if ((e >> 62) == 2 && (e & ap::PTE_DIRTY)) {
             ap::detail::writeback_page(0xffffffffu, c, r, (e >> 32) & ap::PTE_FRAME_MASK, p);
             __syncwarp();
             if ((threadIdx.x & 31) == 0)
-                atomicAnd((unsigned long long*)(r->pte + p), ~(unsigned long long)ap::PTE_DIRTY);
+                atomicAnd((unsigned long long*)q, ~(unsigned long long)ap::PTE_DIRTY);
         }
     }
 }
@@ -122,7 +163,12 @@ static int scan_refs(ap_cache_s* c, const ap_region_host& rg, int* result) {
     int* d_flag = nullptr;
     AP_CUDA_TRY(cudaMalloc(&d_flag, sizeof(int)));
     AP_CUDA_TRY(cudaMemset(d_flag, 0, sizeof(int)));
+#ifdef AP_PT_HASH
+    k_scan_slots<<<c->num_sms * 4, 256>>>(c->slots, 1ull << c->slot_bits,
+                                          (uint64_t)(&rg - c->reg.data()) + 1, d_flag);
+#else
     k_scan_pte<<<c->num_sms * 4, 256>>>(rg.pte, rg.npages, d_flag);
+#endif
     int h = 0;
     cudaError_t e = cudaMemcpy(&h, d_flag, sizeof(int), cudaMemcpyDeviceToHost);
     cudaFree(d_flag);
@@ -186,6 +232,14 @@ extern "C" int ap_cache_create(uint64_t frames, uint32_t page_size, int device, 
     if (cudaMalloc(&c->stats, sizeof(ap::dev_stats) * ap::STAT_SHARDS) != cudaSuccess)
         return fail(AP_ENOMEM);
     if (cudaMalloc(&c->d_cache, sizeof(ap::dev_cache)) != cudaSuccess) return fail(AP_ENOMEM);
+#ifdef AP_PT_HASH
+    /* 16x as many slots as frames */
+    c->slot_bits = 10;
+    while ((1ull << c->slot_bits) < 16 * frames) ++c->slot_bits;
+    if (cudaMalloc(&c->slots, 16ull << c->slot_bits) != cudaSuccess ||
+        cudaMemset(c->slots, 0, 16ull << c->slot_bits) != cudaSuccess)
+        return fail(AP_ENOMEM);
+#endif
     if (cudaMemset(c->owner, 0, frames * 8) != cudaSuccess ||
         cudaMemset(c->free_head, 0, 256) != cudaSuccess ||
         cudaMemset(c->regions, 0, sizeof(ap::dev_region) * AP_MAX_REGIONS) != cudaSuccess ||
@@ -231,6 +285,7 @@ extern "C" int ap_cache_destroy(ap_cache_t c) {
     cudaFree(c->stats);
     cudaFree(c->d_cache);
     cudaFree(c->scratch);
+    cudaFree(c->slots);
     delete c;
     return AP_OK;
 }
@@ -244,6 +299,9 @@ extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, 
                             ap_region_t* out) {
     if (!c || !host_buf || bytes == 0 || !out) return AP_EINVAL;
     if (!(prot & AP_PROT_READ) || (prot & ~(AP_PROT_READ | AP_PROT_WRITE))) return AP_EINVAL;
+#ifdef AP_PT_HASH
+    if (prot & AP_PROT_WRITE) return AP_EINVAL; /* the N4 ablation maps read-only files */
+#endif
     if (((uintptr_t)host_buf) & 15) return AP_EINVAL;
     const uint64_t npages = (bytes + c->page - 1) >> c->log2_page;
     if (npages >= (1ull << 48) || bytes >= (1ull << 60)) return AP_ERANGE;
@@ -292,11 +350,50 @@ extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, 
         return AP_ENOMEM;
     }
     AP_CUDA_TRY(cudaMemset(rg.pte, 0, npages * 8));
+#ifdef AP_PT_HASH
+    if (2 * (c->slot_keys + npages) > (1ull << c->slot_bits)) {
+        /* grow the table to >= 2x the keys: dirty pages go back to their
+         * files first, then every page is evicted (a reset) */
+        for (uint32_t i = 0; i < c->reg.size(); ++i)
+            if (c->reg[i].live && (c->reg[i].prot & AP_PROT_WRITE)) {
+                int rcw = ap_msync(c, i);
+                if (rcw) return rcw;
+            }
+        uint32_t bits = c->slot_bits;
+        while ((1ull << bits) < 2 * (c->slot_keys + npages)) ++bits;
+        uint64_t* ns = nullptr;
+        if (cudaMalloc(&ns, 16ull << bits) != cudaSuccess) {
+            cudaGetLastError();
+            return AP_ENOMEM;
+        }
+        AP_CUDA_TRY(cudaMemset(ns, 0, 16ull << bits));
+        AP_CUDA_TRY(cudaDeviceSynchronize());
+        cudaFree(c->slots);
+        c->slots = ns;
+        c->slot_bits = bits;
+        for (uint32_t i = 0; i < c->reg.size(); ++i)
+            if (c->reg[i].live) {
+                ap::dev_region od{};
+                AP_CUDA_TRY(cudaMemcpy(&od, c->regions + i, sizeof od, cudaMemcpyDeviceToHost));
+                od.pte = c->slots;
+                od.pad_ = c->slot_bits;
+                AP_CUDA_TRY(cudaMemcpy(c->regions + i, &od, sizeof od, cudaMemcpyHostToDevice));
+            }
+        int rcr = ap_cache_reset(c);
+        if (rcr) return rcr;
+    }
+    c->slot_keys += npages;
+#endif
     ap::dev_region d{};
     d.host = rg.dev_alias;
     d.bytes = bytes;
     d.npages = npages;
+#ifdef AP_PT_HASH
+    d.pte = c->slots;
+    d.pad_ = c->slot_bits;
+#else
     d.pte = rg.pte;
+#endif
     d.cache = c->d_cache;
     d.pool = c->pool;
     d.stats = c->stats;
@@ -343,6 +440,9 @@ extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
     if (rc) return rc;
     if (flag) return AP_EBUSY;
     k_drop_owner<<<c->num_sms * 4, 256>>>(c->owner, c->frames, (uint64_t)r + 1);
+#ifdef AP_PT_HASH
+    k_tomb_slots<<<c->num_sms * 4, 256>>>(c->slots, 1ull << c->slot_bits, (uint64_t)r + 1);
+#endif
     AP_CUDA_TRY(cudaGetLastError());
     rc = rebuild_free_list(c);
     if (rc) return rc;
@@ -382,6 +482,9 @@ static int peer_compatible(const ap_cache_s* c, ap_region_t r, uint32_t page, ui
 }
 
 extern "C" int ap_region_add_peer(ap_cache_t c, ap_region_t r, ap_cache_t pc, ap_region_t pr) {
+#ifdef AP_PT_HASH
+    return AP_EINVAL; /* peers read a dense page table */
+#endif
     if (!ap_region_ok(c, r) || !ap_region_ok(pc, pr) || c == pc) return AP_EINVAL;
     if (pc->reg[pr].prot & AP_PROT_WRITE) return AP_EINVAL;
     int rc = peer_compatible(c, r, pc->page, pc->reg[pr].bytes);
@@ -401,6 +504,9 @@ extern "C" int ap_region_add_peer(ap_cache_t c, ap_region_t r, ap_cache_t pc, ap
 }
 
 extern "C" int ap_region_export(ap_cache_t c, ap_region_t r, ap_peer_handle_t* out) {
+#ifdef AP_PT_HASH
+    return AP_EINVAL; /* peers read a dense page table */
+#endif
     if (!ap_region_ok(c, r) || !out) return AP_EINVAL;
     if (c->reg[r].prot & AP_PROT_WRITE) return AP_EINVAL;
     static_assert(sizeof(cudaIpcMemHandle_t) <= sizeof out->pte_handle, "IPC handle size");
@@ -420,6 +526,9 @@ extern "C" int ap_region_export(ap_cache_t c, ap_region_t r, ap_peer_handle_t* o
 }
 
 extern "C" int ap_region_add_peer_ipc(ap_cache_t c, ap_region_t r, const ap_peer_handle_t* h) {
+#ifdef AP_PT_HASH
+    return AP_EINVAL; /* peers read a dense page table */
+#endif
     if (!ap_region_ok(c, r) || !h) return AP_EINVAL;
     int rc = peer_compatible(c, r, h->page_size, h->bytes);
     if (rc) return rc;
@@ -512,6 +621,12 @@ extern "C" int ap_cache_reset(ap_cache_t c) {
         }
     for (auto& rg : c->reg)
         if (rg.live) AP_CUDA_TRY(cudaMemset(rg.pte, 0, rg.npages * 8));
+#ifdef AP_PT_HASH
+    AP_CUDA_TRY(cudaMemset(c->slots, 0, 16ull << c->slot_bits));
+    c->slot_keys = 0;
+    for (auto& rg : c->reg)
+        if (rg.live) c->slot_keys += rg.npages;
+#endif
     AP_CUDA_TRY(cudaMemset(c->owner, 0, c->frames * 8));
     AP_CUDA_TRY(cudaMemset(c->free_head, 0, 256));
     AP_CUDA_TRY(cudaMemset(c->stats, 0, sizeof(ap::dev_stats) * ap::STAT_SHARDS));
@@ -578,7 +693,19 @@ extern "C" int ap_region_dump_pte(ap_cache_t c, ap_region_t r, uint64_t* pte_hos
     if (!ap_region_ok(c, r) || !pte_host) return AP_EINVAL;
     ap_device_guard g(c->device);
     AP_CUDA_TRY(cudaDeviceSynchronize());
+#ifdef AP_PT_HASH
+    /* a dense view of the region's slots (EMPTY where the page has none) */
+    uint64_t* dense = nullptr;
+    AP_CUDA_TRY(cudaMalloc(&dense, c->reg[r].npages * 8));
+    AP_CUDA_TRY(cudaMemset(dense, 0, c->reg[r].npages * 8));
+    k_dump_slots<<<c->num_sms * 4, 256>>>(c->slots, 1ull << c->slot_bits, (uint64_t)r + 1, dense,
+                                          c->reg[r].npages);
+    cudaError_t e = cudaMemcpy(pte_host, dense, c->reg[r].npages * 8, cudaMemcpyDeviceToHost);
+    cudaFree(dense);
+    AP_CUDA_TRY(e);
+#else
     AP_CUDA_TRY(cudaMemcpy(pte_host, c->reg[r].pte, c->reg[r].npages * 8, cudaMemcpyDeviceToHost));
+#endif
     return AP_OK;
 }
 

@@ -1,0 +1,34 @@
+"""N4 ablation: the paper's hash-table page table (one
+concurrent hash table for the pages of all files, 16x the frames, lock-free
+reads) built as libapointer_hash.so (-DAP_PT_HASH).  The read and collage
+parity suites run against it in a subprocess (the binding loads one library
+per process, AP_LIB_PATH selects it): every value must still equal the
+oracle and every page-cache invariant must hold.  The ablation maps
+read-only files only (writable mappings return AP_EINVAL there)."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+LIB = os.path.join(ROOT, "paper_conf_isca_shaharbs16_b200", "libapointer_hash.so")
+
+
+@pytest.mark.xfail(reason="open: under concurrent eviction the hash build occasionally leaks a "
+                          "reference count or faults on a stale frame (the dense build, the "
+                          "product, is clean); see DESIGN.md §10", strict=False)
+def test_hash_page_table_passes_the_parity_suites():
+    assert os.path.exists(LIB), "build libapointer_hash.so (make)"
+    env = dict(os.environ, AP_LIB_PATH=LIB)
+    probe = subprocess.run([sys.executable, "-c",
+                            "import paper_conf_isca_shaharbs16_b200 as ap; print(ap.ap_version())"],
+                           cwd=ROOT, env=env, capture_output=True, text=True, timeout=300)
+    assert "hash-table page table" in probe.stdout, probe.stdout + probe.stderr
+    r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
+                        "tests/test_gpu_reads.py", "tests/test_gpu_collage.py"],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=1500)
+    assert r.returncode == 0, r.stdout[-4000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout
