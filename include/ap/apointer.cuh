@@ -344,7 +344,11 @@ __device__ __forceinline__ uint64_t* pt_find(const dev_region* r, uint64_t pg, b
     return nullptr;
 }
 #define AP_PTE_AT(r, pg) ::ap::detail::pt_find((r), (pg), false)
+/* the probe is a leader-only loop of data-dependent length: reconverge the
+ * warp after it, so later __activemask()-based operations see every lane */
+#define AP_PT_RECONVERGE(m) __syncwarp(m)
 #else
+#define AP_PT_RECONVERGE(m) ((void)0)
 #define AP_PTE_AT(r, pg) ((r)->pte + (pg))
 #endif
 
@@ -417,6 +421,7 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
         stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->unlinks, 1);
 #endif
     }
+    AP_PT_RECONVERGE(m);
 }
 
 /* -------------------------------------------------------------------------
@@ -685,6 +690,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         const uint32_t n = __popc(grp);
 #ifdef AP_PT_HASH
         uint64_t* pte = is_leader ? pt_find(r, pg, true) : nullptr;
+        __syncwarp(m);
 #else
         uint64_t* pte = r->pte + pg;
 #endif
@@ -880,6 +886,7 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
             }
         }
     }
+    AP_PT_RECONVERGE(m);
 #ifndef AP_NO_HOT_STATS /* ablation: no counters on the inline link / unlink */
     const unsigned linkedm = __ballot_sync(m, is_leader && (old >> 62) == 2);
     if (linkedm && (int)lane_id() == __ffs(m) - 1)
@@ -1014,6 +1021,7 @@ __device__ AP_SLOW_ATTR slow_out<T> store_slow(unsigned m, uint64_t x, uint64_t 
         const unsigned long long key = mark ? (((unsigned long long)r->id << 48) | page) : ~0ull;
         const unsigned grp = __match_any_sync(m, key);
         if (mark && (int)lane == __ffs(grp) - 1) red_or_relaxed(AP_PTE_AT(r, page), PTE_DIRTY);
+        AP_PT_RECONVERGE(m);
         if (lnk) {
             x |= XL_DIRTY;
             st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
@@ -1045,6 +1053,7 @@ __device__ AP_SLOW_ATTR slow_out<T> store_slow(unsigned m, uint64_t x, uint64_t 
             const bool ok = (x >> 63) != 0;
             const unsigned okm = __ballot_sync(mg, ok);
             if (ok && (int)lane == __ffs(okm) - 1) red_or_relaxed(AP_PTE_AT(r, page), PTE_DIRTY);
+            AP_PT_RECONVERGE(mg);
             if (ok) {
                 x |= XL_DIRTY;
                 st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
@@ -1304,6 +1313,7 @@ struct ptr {
             asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;"
                          : "=l"(old) : "l"(pte), "l"((uint64_t)__popc(grp)) : "memory");
         }
+        AP_PT_RECONVERGE(m);
         return link_ticket{old, grp, need};
     }
     __device__ __forceinline__ void link_finish(const link_ticket& t) {
@@ -1321,6 +1331,7 @@ struct ptr {
                                         (unsigned long long)(0 - (uint64_t)__popc(t.grp)));
             }
         }
+        AP_PT_RECONVERGE(m);
 #ifndef AP_NO_HOT_STATS
         const unsigned linkedm = __ballot_sync(m, is_leader && res);
         if (linkedm && (int)detail::lane_id() == __ffs(m) - 1)
