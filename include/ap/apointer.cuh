@@ -343,11 +343,27 @@ __device__ __forceinline__ uint64_t* pt_find(const dev_region* r, uint64_t pg, b
     }
     return nullptr;
 }
+#ifdef AP_PT_HASH_DIAG
+/* diagnostic: a must-exist lookup that finds no slot sets ERR_FAULT and
+ * hands out a scratch counter word instead of crashing */
+__device__ __forceinline__ uint64_t* pt_must(const dev_region* r, uint64_t pg) {
+    uint64_t* q = pt_find(r, pg, false);
+    if (!q) {
+        atomicCAS(r->cache->err, 0, ERR_FAULT - 100);
+        return reinterpret_cast<uint64_t*>(&r->stats->waits);
+    }
+    return q;
+}
+#define AP_PTE_AT(r, pg) ::ap::detail::pt_must((r), (pg))
+#else
 #define AP_PTE_AT(r, pg) ::ap::detail::pt_find((r), (pg), false)
+#endif
 /* the probe is a leader-only loop of data-dependent length: reconverge the
  * warp after it, so later __activemask()-based operations see every lane */
+#define AP_PTE_FIND(r, pg) ::ap::detail::pt_find((r), (pg), false) /* may miss */
 #define AP_PT_RECONVERGE(m) __syncwarp(m)
 #else
+#define AP_PTE_FIND(r, pg) ((r)->pte + (pg))
 #define AP_PT_RECONVERGE(m) ((void)0)
 #define AP_PTE_AT(r, pg) ((r)->pte + (pg))
 #endif
@@ -505,7 +521,7 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         const uint64_t own = ld_relaxed(c->owner + f);
         if (own) {
             const dev_region* vr = c->regions + ((own >> 48) - 1);
-            q = AP_PTE_AT(vr, own & PAGE_MASK48);
+            q = AP_PTE_FIND(vr, own & PAGE_MASK48);
 #ifdef AP_PT_HASH
             /* the owner entry can become visible before the key's insert */
             e = q ? ld_relaxed(q) : 0;
@@ -555,7 +571,7 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
 #ifdef AP_DEBUG
     if (still && (int)lane == first) {
         const uint64_t own0 = ld_relaxed(c->owner);
-        const uint64_t* q0 = own0 ? AP_PTE_AT(&c->regions[(own0 >> 48) - 1], own0 & PAGE_MASK48) : nullptr;
+        const uint64_t* q0 = own0 ? AP_PTE_FIND(&c->regions[(own0 >> 48) - 1], own0 & PAGE_MASK48) : nullptr;
         const uint64_t e0 = q0 ? ld_relaxed(q0) : 0;
         if ((clock64() & 0xfffff) < 200)
             printf("[nofree] sm %u warp %u m %08x own0 %llx e0 %llx hand %llu\n", sm_id(),
@@ -1305,7 +1321,7 @@ struct ptr {
             __match_any_sync(m, need ? (((unsigned long long)r->id << 48) | pg) : ~0ull);
         uint64_t old = 0;
         if (need && (int)detail::lane_id() == __ffs(grp) - 1) {
-            uint64_t* pte = AP_PTE_AT(r, pg);
+            uint64_t* pte = AP_PTE_FIND(r, pg);
 #ifdef AP_PT_HASH
             if (!pte) old = 3ull << 62; /* no slot: nothing added (no early return: */
             else                        /* the warp must stay converged)            */

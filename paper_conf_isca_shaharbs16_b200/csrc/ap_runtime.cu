@@ -145,7 +145,7 @@ __global__ void k_writeback(const ap::dev_cache* __restrict__ c, uint32_t region
     const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) / 32;
     const uint64_t nwarps = (uint64_t)gridDim.x * blockDim.x / 32;
     for (uint64_t p = warp; p < r->npages; p += nwarps) {
-        uint64_t* q = AP_PTE_AT(r, p);
+        uint64_t* q = AP_PTE_FIND(r, p);
 #ifdef AP_PT_HASH
         if (!q) continue;
 #endif
