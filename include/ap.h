@@ -242,6 +242,7 @@ typedef struct {
 #define AP_ACCESS_RANGE 2
 #define AP_ACCESS_AHEAD 3 /* TILE + the next unit linked split-phase under the last tile */
 #define AP_ACCESS_PAIR 4  /* TILE over two units whose links are issued together */
+#define AP_ACCESS_TMA 5   /* 16-B checksums staged through shared memory by TMA bulk copies */
 
 /* Run one microbenchmark launch (asynchronous on `stream`).
  * out_dev: uint64[grid*block] per-thread FNV-1a-64 checksums over the values

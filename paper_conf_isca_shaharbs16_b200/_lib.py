@@ -15,7 +15,7 @@ AP_EFAULT, AP_ENOFRAME, AP_ETIMEDOUT = -6, -7, -8
 AP_POLICY_CLOCK, AP_POLICY_RANDOM = 0, 1
 AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
-AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_AHEAD, AP_ACCESS_PAIR = 0, 1, 2, 3, 4
+AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_AHEAD, AP_ACCESS_PAIR, AP_ACCESS_TMA = 0, 1, 2, 3, 4, 5
 AP_SCHED_NATURAL, AP_SCHED_LSH, AP_SCHED_TABLE, AP_SCHED_TABLE_MH = 0, 1, 2, 3
 AP_PROT_READ, AP_PROT_WRITE = 1, 2
 AP_EPERM = -9

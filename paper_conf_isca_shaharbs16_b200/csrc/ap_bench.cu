@@ -331,6 +331,93 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     if (!a.out_copy) a.ck[t] = h;
 }
 
+/* AP_ACCESS_TMA (16-B elements, checksums): the SEQ stream staged through
+ * shared memory with TMA bulk copies (cp.async.bulk + mbarrier) instead of a
+ * register tile: TMA_ST stages of TMA_SB bytes per warp (12 KiB in flight
+ * per warp, 192 KiB per CTA of 16 warps) and no loaded value in registers.
+ * Apointer: each unit is pinned once (pin_range, a minor fault when
+ * resident) when its first stage is issued and unlinked when its last stage
+ * has been consumed, so the next unit's link overlaps the stages still in
+ * flight (two units live at most: ptr[unit & 1]).  The raw twin runs the
+ * same loop from a plain pointer.  Consumption order = the tiled kernel's,
+ * so the checksums are identical. */
+constexpr int TMA_ST = 6;
+constexpr uint32_t TMA_SB = 2048;
+constexpr int TMA_WARPS = AP_BENCH_THREADS / 32;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+template <bool APTR>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, 1)
+    k_seq_tma(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
+    extern __shared__ __align__(128) uint8_t tma_smem[];
+    __shared__ __align__(8) uint64_t mbar[TMA_WARPS][TMA_ST];
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const unsigned wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint64_t w = t >> 5;
+    const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t nunits = a.span / a.unit;
+    const uint32_t spu = a.unit / TMA_SB; /* stages per unit */
+    uint8_t* buf = tma_smem + (size_t)wid * TMA_ST * TMA_SB;
+    uint64_t h = FNV_BASIS;
+    if (lane == 0) {
+        for (int b = 0; b < TMA_ST; ++b)
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[wid][b])));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    const uint64_t per_warp = w < nunits ? (nunits - w + W - 1) / W : 0;
+    const uint64_t total = per_warp * a.passes * spu; /* stages of this warp */
+    [[maybe_unused]] ap::ptr<uint4> q[2];
+    const uint8_t* ubase[2] = {nullptr, nullptr};
+    auto issue = [&](uint64_t g) {
+        const uint64_t k = g / spu, st = g % spu;
+        const uint64_t u = w + (k % per_warp) * W;
+        if (st == 0) {
+            if constexpr (APTR) {
+                q[k & 1] = ap::gvmmap<uint4>(c, region, u * a.unit);
+                const uint4* p = q[k & 1].pin_range(a.unit);
+                ubase[k & 1] = reinterpret_cast<const uint8_t*>(p);
+                /* frame data written by the generic proxy (fills), read by
+                 * the async proxy (TMA) */
+                asm volatile("fence.proxy.async.global;" ::: "memory");
+            } else {
+                ubase[k & 1] = a.raw + u * a.unit;
+            }
+        }
+        if (lane == 0) {
+            const uint32_t mb = smem_u32(&mbar[wid][g % TMA_ST]);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb),
+                         "r"(TMA_SB) : "memory");
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                ::"r"(smem_u32(buf + (g % TMA_ST) * TMA_SB)), "l"(ubase[k & 1] + st * TMA_SB),
+                "r"(TMA_SB), "r"(mb) : "memory");
+        }
+    };
+    for (uint64_t g = 0; g < total && g < (uint64_t)TMA_ST; ++g) issue(g);
+    for (uint64_t g = 0; g < total; ++g) {
+        const int b = (int)(g % TMA_ST);
+        const uint32_t parity = (uint32_t)((g / TMA_ST) & 1);
+        const uint32_t mb = smem_u32(&mbar[wid][b]);
+        uint32_t done = 0;
+        while (!done)
+            asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                         : "=r"(done) : "r"(mb), "r"(parity) : "memory");
+        const uint4* sv = reinterpret_cast<const uint4*>(buf + b * TMA_SB);
+#pragma unroll
+        for (int jj = 0; jj < (int)(TMA_SB / 512); ++jj) h = fnv(h, sv[jj * 32 + lane]);
+        __syncwarp();
+        if constexpr (APTR) {
+            if (g % spu == spu - 1) q[(g / spu) & 1].release(); /* unit consumed */
+        }
+        if (g + TMA_ST < total) issue(g + TMA_ST);
+    }
+    a.ck[t] = h;
+}
+
 /* ------------------------------------------------------------ UNIFORM / DIVERGENT */
 template <class T, int PAT, bool APTR>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_BENCH_MINB)
@@ -369,6 +456,13 @@ cudaError_t launch_t(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg
                 k_seq_deref<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             else if (APTR && (cfg->access == AP_ACCESS_AHEAD || cfg->access == AP_ACCESS_PAIR))
                 k_seq_split<T><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            else if (cfg->access == AP_ACCESS_TMA) {
+                if constexpr (sizeof(T) == 16) {
+                    const int smem = TMA_WARPS * TMA_ST * (int)TMA_SB;
+                    cudaFuncSetAttribute(k_seq_tma<APTR>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                    k_seq_tma<APTR><<<cfg->grid, cfg->block, smem, s>>>(c->d_cache, region, a);
+                }
+            }
             else
                 k_seq<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             break;
@@ -412,13 +506,19 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
     a->page = cfg->page_bytes;
     a->span = cfg->span_bytes ? cfg->span_bytes : rg.bytes;
     a->access = cfg->access;
-    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_PAIR) return AP_EINVAL;
+    if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_TMA) return AP_EINVAL;
     switch (cfg->pattern) {
         case AP_SEQ:
             if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;
             if (cfg->mode == AP_MODE_APOINTER && (c->page % a->unit)) return AP_EINVAL;
             if (cfg->out_copy) a->out_copy = (uint8_t*)out;
             else a->ck = (uint64_t*)out;
+            /* TMA staging: 16-B checksums over whole units of whole stages,
+             * at least as many stages per unit as are in flight */
+            if (cfg->access == AP_ACCESS_TMA &&
+                (E != 16 || cfg->out_copy || a->unit % TMA_SB || a->unit / TMA_SB < TMA_ST ||
+                 a->span % a->unit || cfg->block > AP_BENCH_THREADS))
+                return AP_EINVAL;
             break;
         case AP_UNIFORM: /* offsets uniform over [0, span) (span 0 = the region) */
             if (a->span < E || a->span > rg.bytes) return AP_EINVAL;

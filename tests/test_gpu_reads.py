@@ -253,3 +253,39 @@ def test_per_access_deref_kernel(ap, dev, frames):
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("prefill,frames,unit", [(True, 1024, 65536), (False, 24, 16384),
+                                                 (False, 3, 65536)])
+def test_seq_tma_staged(ap, dev, prefill, frames, unit):
+    """AP_ACCESS_TMA: the SEQ stream staged through shared memory by TMA bulk
+    copies, one pin per unit; apointer and raw twin == oracle, resident or
+    faulting (3 frames: every unit evicts, two units pinned per warp at most)."""
+    page, nbytes = 65536, 16 << 20
+    f = make_file(nbytes, seed=41)
+    cache = ap.ap_cache_create(frames, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        if prefill:
+            ap.ap_prefill(cache, r, 0, min(frames, nbytes // page))
+            torch.cuda.synchronize()
+        grid, block = (148, 512) if frames > 3 else (1, 32)
+        cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=2,
+                           access=ap.AP_ACCESS_TMA)
+        got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+        want = oracle.read_seq(f, nbytes, unit, 16, grid * block, 2)
+        assert np.array_equal(got, want)
+        dcopy = torch.from_numpy(f).to(dev)
+        cfg_raw = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=2,
+                               access=ap.AP_ACCESS_TMA, mode=ap.AP_MODE_RAW,
+                               raw_base=dcopy.data_ptr())
+        assert np.array_equal(_run(ap, cache, r, cfg_raw, grid * block, dev).view(np.uint64), want)
+        assert check_invariants(ap, cache, [r], frames) == []
+        from paper_conf_isca_shaharbs16_b200._lib import APError
+        with pytest.raises(APError):  # 4-B elements are not staged
+            ap.ap_bench_read(cache, r, ap.bench_cfg(ap.AP_SEQ, 4, 1, 32, unit_bytes=unit,
+                                                    access=ap.AP_ACCESS_TMA),
+                             torch.zeros(32, dtype=torch.int64, device=dev))
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)

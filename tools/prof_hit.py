@@ -51,6 +51,17 @@ def t(fn, n=5):
 
 tr = t(lambda: ap.ap_bench_read(cache, r, cfg_raw, out2))
 nb = span * passes
+cfg_traw = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=passes, span_bytes=span,
+                        mode=ap.AP_MODE_RAW, raw_base=dcopy.data_ptr(), access=ap.AP_ACCESS_TMA)
+cfg_tap = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=passes, span_bytes=span,
+                       access=ap.AP_ACCESS_TMA)
+out3 = torch.empty_like(out)
+for _ in range(3):
+    ttr = t(lambda: ap.ap_bench_read(cache, r, cfg_traw, out3))
+    tta = t(lambda: ap.ap_bench_read(cache, r, cfg_tap, out))
+    print(f"unit={unit} passes={passes} tma   apointer {span * passes / tta[1] / 1e9:.1f} GB/s raw-tma "
+          f"{span * passes / ttr[1] / 1e9:.1f} GB/s overhead {tta[1] / ttr[1] - 1:.3f} "
+          f"(vs tiled raw {tta[1] / tr[1] - 1:+.3f}) equal={bool(torch.equal(out, out2)) and bool(torch.equal(out3, out2))}")
 for acc, name in ((ap.AP_ACCESS_TILE, "tile"), (ap.AP_ACCESS_AHEAD, "ahead"), (ap.AP_ACCESS_PAIR, "pair"), (ap.AP_ACCESS_RANGE, "range"), (ap.AP_ACCESS_DEREF, "deref")):
     cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=passes, span_bytes=span,
                        access=acc)
