@@ -430,7 +430,18 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
 #ifdef AP_DEBUG
         printf("[unlink] w%u m%08x grp%08x n%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, grp, n, (unsigned long long)page);
 #endif
+#ifdef AP_PT_HASH_DIAG
+        {
+            /* diagnostic: an unlink must find its page VALID with a count >= n */
+            uint64_t* q = AP_PTE_AT(r, page);
+            const unsigned long long o = atomicAdd(reinterpret_cast<unsigned long long*>(q),
+                                                   (unsigned long long)(0 - (uint64_t)n));
+            if ((o >> 62) != 2 || (o & PTE_RC_MASK) < n)
+                atomicCAS(r->cache->err, 0, (o >> 62) != 2 ? -107 : -108);
+        }
+#else
         red_unlink(AP_PTE_AT(r, page), (uint64_t)0 - (uint64_t)n);
+#endif
 #if defined(AP_COUNT_UNLINKS) && !defined(AP_NO_HOT_STATS)
         /* opt-in: one more atomic per unlink cost a third of the minor-fault
          * throughput (M2r 14.5 -> 10.0 G reads/s), so it is off by default */
