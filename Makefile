@@ -9,8 +9,15 @@ HOSTCC  := $(shell test -x /usr/bin/gcc && echo /usr/bin/gcc || echo gcc)
 PKG     := paper_conf_isca_shaharbs16_b200
 CSRC    := $(PKG)/csrc
 ARCH    := -gencode arch=compute_100a,code=sm_100a
+# -rdc=true: the out-of-line fault path (deref_slow and friends) is called
+# through the ABI, so values a hot loop keeps live across a possible fault stay
+# in callee-saved registers and are saved only inside the fault path (a
+# whole-program call made ptxas spill them at their definition, on the hit
+# path).  -maxrregcount=64 sizes those ABI functions for every caller (the
+# paper's 64 registers per thread); kernels keep their own
+# __launch_bounds__ budgets.
 NVFLAGS := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -Wall \
-           -Iinclude -I$(CSRC) --expt-relaxed-constexpr
+           -Iinclude -I$(CSRC) --expt-relaxed-constexpr -rdc=true -maxrregcount=64
 CFLAGS  := -O2 -fopenmp -fPIC -Wall -Wextra -std=c11
 
 CU_SRCS := $(wildcard $(CSRC)/*.cu)

@@ -78,7 +78,8 @@ def _shm_records(cfg, rank, world, dist):
     return np.frombuffer(mm, dtype=np.uint8), (fh, mm)
 
 
-def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_link_peak):
+def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_link_peak,
+                light=False):
     import paper_conf_isca_shaharbs16_b200 as ap
     import synth
     cfg = collage_config(args.workload, args.stride)
@@ -168,7 +169,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     got = win.cpu().numpy().view(np.uint32).copy()
     # the other schedules, for comparison (cold cache, same winners)
     other_res = []
-    for other in (s for s in (0, 1, 2, 3) if s != args.schedule and world == 1):
+    for other in (s for s in (0, 1, 2, 3) if s != args.schedule and world == 1 and not light):
         inp_o = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                               cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
                               block_count=b1 - b0, schedule=other)
@@ -207,6 +208,14 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         npages = (cfg["N"] * cfg["stride"] + cfg["page"] - 1) // cfg["page"]
         big = ap.ap_cache_create(npages + 64, cfg["page"], torch.cuda.current_device())
         rb = ap.ap_mmap(big, recs)
+        # one cold run on a cache that holds every record: its major faults
+        # are the distinct record pages this rank's share touches, the
+        # host-link lower bound of a cold step (each needed page read once)
+        wd = torch.empty_like(win)
+        ap.ap_collage_run(big, rb, inp, wd, stream)
+        torch.cuda.synchronize()
+        raw_distinct = ap.ap_cache_stats(big)["major"]
+        ap.ap_cache_reset(big)
         ap.ap_prefill(big, rb, 0, npages, stream)
         torch.cuda.synchronize()
         res_g = {}
@@ -230,6 +239,8 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
                             equal=bool(torch.equal(wg, win) and torch.equal(wr, win)))
         raw["resident"] = res_g
         raw["resident_majors"] = ap.ap_cache_stats(big)["major"]
+        raw["distinct_pages"] = raw_distinct
+        raw["distinct_equal"] = bool(torch.equal(wd, win))
         ap.ap_munmap(big, rb)
         ap.ap_cache_destroy(big)
         del dcopy
@@ -262,40 +273,40 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     if bucket and rank == 0:
         got = full.cpu().numpy().view(np.uint32).copy()  # rank 0's own array is partial
         res["got"] = got
-    if rank == 0 and full is not None and not args.no_cpu_baseline:
+    po = pi = None
+    if rank == 0 and not args.no_cpu_baseline:
+        # the oracle's own bucket index (never the GPU-built CSR): the oracle
+        # collage runs on it, and the GPU index must equal it
         import oracle
+        t0 = time.time()
+        po, pi = oracle.build_index(recs, cfg["stride"], cfg["N"], proj, bias, cfg["w"], cfg["bb"],
+                                    threads=os.cpu_count() or 1)
+        t_oindex = time.time() - t0
+        index_equal = bool(np.array_equal(po, off.cpu().numpy().view(np.uint32)) and
+                           np.array_equal(pi, ids.cpu().numpy().view(np.uint32)))
+    if rank == 0 and full is not None and not args.no_cpu_baseline:
         fw = full.cpu().numpy().view(np.uint32)
-        o_off = off.cpu().numpy().view(np.uint32)
-        o_ids = ids.cpu().numpy().view(np.uint32)
         ok = True
         for r_ in range(world):  # 16 blocks from the start of every rank's range
             rb0, rb1 = mgpu.block_range(nb, r_, world)
             k = min(16, rb1 - rb0)
             want = oracle.collage(img, proj, bias, cfg["w"], cfg["bb"], recs, cfg["stride"],
-                                  cfg["N"], o_off, o_ids, b0=rb0, nb=k,
-                                  threads=os.cpu_count() or 1)
+                                  cfg["N"], po, pi, b0=rb0, nb=k, threads=os.cpu_count() or 1)
             ok = ok and bool(np.array_equal(want, fw[rb0:rb0 + k]))
         res["gathered_parity"] = dict(ranks=world, blocks_per_rank=16, equal=ok,
                                       partition=("records (id slices)" if i1 else "buckets (units)")
                                       if bucket else "blocks")
     if rank == 0 and not args.no_cpu_baseline:
-        import oracle
-        o_off = off.cpu().numpy().view(np.uint32)
-        o_ids = ids.cpu().numpy().view(np.uint32)
         threads = os.cpu_count() or 1
         nsample = (b1 - b0) if cfg["name"] == "c4" else min(256, b1 - b0)
         t0 = time.time()
         want = oracle.collage(img, proj, bias, cfg["w"], cfg["bb"], recs, cfg["stride"], cfg["N"],
-                              o_off, o_ids, b0=b0, nb=nsample, threads=threads)
+                              po, pi, b0=b0, nb=nsample, threads=threads)
         dt = time.time() - t0
         res["parity"] = dict(blocks=nsample, equal=bool(np.array_equal(want, got[:nsample])),
-                             cpu_s=dt, cores=threads)
-        # the index itself vs the oracle's (c4: full; c5: skipped, 10M records)
-        if cfg["name"] == "c4":
-            po, pi = oracle.build_index(recs, cfg["stride"], cfg["N"], proj, bias, cfg["w"],
-                                        cfg["bb"], threads=threads)
-            res["parity"]["index_equal"] = bool(np.array_equal(po, o_off) and
-                                                np.array_equal(pi, o_ids))
+                             cpu_s=dt, cores=threads, index_equal=index_equal,
+                             oracle_index_s=round(t_oindex, 2),
+                             empty_blocks=int(np.all(want == oracle.EMPTY, axis=1).sum()))
     ap.ap_munmap(cache, region)
     ap.ap_cache_destroy(cache)
     if keep:
@@ -392,3 +403,51 @@ def emit_collage(args, res_all, world, METRIC):
                                 "sample": f"oracle collage over {p['blocks']} of rank 0's "
                                           f"{full_blocks} blocks, scaled to all of them"}
     return line
+
+
+def collage_summary(args, res_all, world):
+    """The C4 collage object embedded in the default bench line (BASELINE.json
+    configs[3]): seconds per cold step (max over ranks),
+    its spread, fills, the host-link bound of the distinct records, the
+    resident-cache apointer vs raw-twin overhead, parity and the oracle."""
+    r0 = res_all[0]
+    cfg = r0["cfg"]
+    per_rank = [float(np.mean(r["times"])) for r in res_all]
+    tmax = max(per_rank)
+    st = r0["stats"][-1]
+    t = np.asarray(r0["times"]) * 1e3
+    out = {
+        "workload": cfg["workload"], "schedule": SCHED_NAMES[args.schedule],
+        "group": args.group, "id_chunks": r0["id_chunks"],
+        "parallelism": ("record-id slices over %d ranks" % world) if r0.get("records") else
+                       ("units over %d ranks" % world) if r0.get("bucket") else
+                       ("blocks over %d rank(s)" % world),
+        "s": round(tmax, 6), "per_rank_s": [round(x, 6) for x in per_rank],
+        "step_times": {"mean_ms": round(float(t.mean()), 4),
+                       "std_ms": round(float(t.std(ddof=1)) if len(t) > 1 else 0.0, 4),
+                       "n": int(len(t))},
+        "fill_GB": round(st["fill_bytes"] / 1e9, 4), "major_faults": st["major"],
+        "device_error": r0["err"], "host_link_GBps": round(r0["link"], 2),
+        "fill_frac_of_host_link": round(st["fill_bytes"] / float(np.mean(r0["times"])) / 1e9 /
+                                        r0["link"], 4),
+        "e2e_s": round(max(float(np.mean(r["e2e"])) for r in res_all), 6),
+    }
+    raw = r0.get("raw")
+    if raw:
+        bound = raw["distinct_pages"] * cfg["page"] / (r0["link"] * 1e9)
+        out["distinct_record_pages"] = raw["distinct_pages"]
+        out["distinct_bound_s"] = round(bound, 6)
+        out["frac_of_distinct_bound"] = round(bound / float(np.mean(r0["times"])), 4)
+        out["resident"] = {f"group{g}": {"apointer_ms": round(d["apointer_s"] * 1e3, 4),
+                                         "raw_ms": round(d["raw_s"] * 1e3, 4),
+                                         "overhead": round(d["overhead"], 4), "equal": d["equal"]}
+                           for g, d in raw["resident"].items()}
+    if r0.get("parity"):
+        p = r0["parity"]
+        out["parity_vs_oracle"] = {k: v for k, v in p.items() if k not in ("cpu_s",)}
+        full_blocks = r0["b1"] - r0["b0"]
+        out["oracle_s"] = round(p["cpu_s"] * full_blocks / p["blocks"], 4)
+        out["oracle_cores"] = p["cores"]
+    if r0.get("gathered_parity"):
+        out["gathered_parity_vs_oracle"] = r0["gathered_parity"]
+    return out

@@ -361,7 +361,19 @@ typedef struct {
      * with the same 64-bit MIN reduction as the bucket partition. */
     uint32_t id_begin;
     uint32_t id_end;
+    /* AP_COLLAGE_ACCUMULATE: winners_dev is NOT initialised; every block's
+     * result is folded into it with the 64-bit lexicographic (dist, idx) min
+     * (R-A3), whatever the schedule, so partitions run by other calls, other
+     * caches or other GPUs can accumulate into one winners array (initialise
+     * it once with ap_winners_init).  AP_COLLAGE_SYSTEM: that min is a
+     * system-scope atomic (winners_dev is another GPU's memory reached over
+     * NVLink peer access, or a CUDA IPC mapping shared across processes).
+     * 0 = the default: winners_dev is written from scratch. */
+    uint32_t flags;
 } ap_collage_in;
+
+#define AP_COLLAGE_ACCUMULATE 1u
+#define AP_COLLAGE_SYSTEM 2u
 
 #define AP_SCHED_NATURAL 0
 #define AP_SCHED_LSH 1
@@ -383,6 +395,98 @@ typedef struct {
  * Errors: AP_EINVAL (W/H not multiples of 32, K > 16, group), AP_ECUDA. */
 int ap_collage_run(ap_cache_t cache, ap_region_t records, const ap_collage_in* in,
                    uint32_t* winners_dev, void* stream);
+
+/* ap_winners_init — set nblocks winners to the empty sentinel
+ * (0xFFFFFFFF, 0xFFFFFFFF) (R-A4), the identity of the winners' min, before
+ * partitions accumulate into them (AP_COLLAGE_ACCUMULATE).  Asynchronous. */
+int ap_winners_init(uint32_t* winners_dev, uint64_t nblocks, void* stream);
+
+/* ---------------------------------------- device buffers across processes
+ * One process per GPU (the framework's launch model): a buffer of one
+ * process's GPU is made addressable by the others with CUDA IPC, so their
+ * kernels can combine results into it directly over NVLink (e.g. the
+ * collage winners with AP_COLLAGE_ACCUMULATE | AP_COLLAGE_SYSTEM) -- no
+ * collective in the data path.  ap_ipc_export works on any address inside a
+ * cudaMalloc allocation of the current process; the handle is plain bytes
+ * (send it with any host-side channel, e.g. torch.distributed's object
+ * all-gather).  ap_ipc_import maps it on `device` and returns the same
+ * address inside the mapping; ap_ipc_close unmaps (pass the address
+ * ap_ipc_import returned).  The exporter keeps the buffer alive until every
+ * importer closed it.  Errors: AP_EINVAL, AP_ECUDA. */
+typedef struct {
+    uint8_t handle[64]; /* cudaIpcMemHandle_t of the allocation            */
+    uint64_t offset;    /* the exported address - the allocation's base    */
+    uint64_t bytes;     /* bytes from the exported address to the end      */
+    int32_t device;     /* exporter's device ordinal (informational)       */
+    int32_t pid;        /* exporter's process id (informational)           */
+} ap_ipc_handle_t;
+int ap_ipc_export(const void* dev_ptr, ap_ipc_handle_t* out);
+int ap_ipc_import(const ap_ipc_handle_t* h, int device, void** dev_ptr);
+int ap_ipc_close(void* dev_ptr);
+
+/* ---------------------------------------------- multi-GPU collage (§8(e))
+ * One process drives G partitions of the collage, each on its own GPU with
+ * its own page cache over the SAME pinned host file (read-only, so no
+ * coherence is needed; the file is registered once for all of them).  The
+ * query blocks are independent, so the partitions share
+ * nothing but the winners: every partition's kernel folds its results
+ * straight into the root GPU's winners array over NVLink peer memory
+ * (system-scope 64-bit atomic min, AP_COLLAGE_ACCUMULATE | AP_COLLAGE_SYSTEM)
+ * -- the combine is fused into the kernels' epilogue, no collective runs.
+ * `devices` may repeat an ordinal: partitions sharing a GPU run concurrently
+ * on their own streams (that is how a one-GPU box exercises G > 1). */
+#define AP_MGPU_MAX 16
+#define AP_PART_BLOCKS 0  /* contiguous block ranges (row bands)                  */
+#define AP_PART_RECORDS 1 /* record-id slices: each cache holds one shard of the
+                           * file; every partition runs all units (per-table
+                           * schedules only)                                      */
+#define AP_PART_UNITS 2   /* slices of the (table, bucket)-sorted units          */
+typedef struct ap_mgpu_s* ap_mgpu_t;
+typedef struct {
+    const uint8_t* target_host;  /* W*H*3 uint8 RGB (caller-owned host memory)   */
+    uint32_t W, H, L, K, bucket_bits;
+    int32_t w;
+    const int16_t* proj_host;    /* [L][K][768]                                  */
+    const int32_t* bias_host;    /* [L][K]                                       */
+    uint64_t N;
+    uint32_t rec_stride, group;
+    int32_t schedule;            /* AP_SCHED_*                                    */
+    uint32_t id_chunks;          /* record-id windows per partition (0 = off)     */
+    int32_t partition;           /* AP_PART_*                                     */
+} ap_mgpu_collage_in;
+typedef struct {
+    double seconds;                   /* the step: CUDA events on the root from
+                                       * before the first partition's launch to
+                                       * after the last one's completion (winners
+                                       * combined); cold caches, no host copies  */
+    double part_seconds[AP_MGPU_MAX]; /* each partition's own kernels           */
+    uint64_t fill_bytes[AP_MGPU_MAX]; /* host-link bytes filled per partition    */
+    uint64_t major[AP_MGPU_MAX];
+    int32_t device_error;             /* first sticky device error, or AP_OK     */
+    int32_t nparts;
+} ap_mgpu_report;
+
+/* ap_mgpu_create — G = ngpu partitions on devices[0..G-1] (devices[0] is the
+ * root holding the winners), each a page cache of frames_per_gpu frames of
+ * page_size bytes mapping host_file (bytes, 16-B aligned, caller-owned,
+ * valid until ap_mgpu_destroy).  Enables peer access from every partition's
+ * GPU to the root.  Errors: AP_EINVAL (ngpu outside 1..AP_MGPU_MAX, no peer
+ * access), AP_ENOMEM, AP_ECUDA. */
+int ap_mgpu_create(int ngpu, const int* devices, const void* host_file, uint64_t bytes,
+                   uint64_t frames_per_gpu, uint32_t page_size, ap_mgpu_t* out);
+/* ap_mgpu_collage — one cold collage step over the G partitions: uploads the
+ * target and LSH parameters and builds the bucket index on every GPU when
+ * they differ from the previous call's (not timed), resets every cache, runs
+ * the partitions concurrently, and copies the combined winners
+ * uint32[blocks][2] into winners_host.  rep (optional) receives the timing
+ * and per-partition counters.  Synchronises.  Errors: as ap_collage_run. */
+int ap_mgpu_collage(ap_mgpu_t m, const ap_mgpu_collage_in* in, uint32_t* winners_host,
+                    ap_mgpu_report* rep);
+int ap_mgpu_destroy(ap_mgpu_t m);
+/* One-shot convenience: create, one step, destroy. */
+int ap_collage_mgpu(int ngpu, const int* devices, const void* host_file, uint64_t bytes,
+                    uint64_t frames_per_gpu, uint32_t page_size, const ap_mgpu_collage_in* in,
+                    uint32_t* winners_host, ap_mgpu_report* rep);
 
 /* ap_lsh_build_index — the dataset index ("The dataset images
  * are placed in buckets indexed by the LSH keys derived from their

@@ -161,6 +161,11 @@ struct alignas(128) dev_region {
     const dev_cache* cache; /* owning cache                               */
     const dev_peer* peers;  /* N2: caches a major fault may copy from     */
     uint32_t npeers;        /* 0 = fills come from the host only          */
+    uint32_t shared;        /* N2: another cache (GPU) pins this region's
+                             * pages as its peer, so the fault path's claim,
+                             * publish and eviction RMWs on these PTEs are
+                             * system-scope (they race with the peer's .sys
+                             * pin, R-A15b)                                */
 };
 
 /* Cache descriptor, one copy in device memory per ap_cache_t. */
@@ -291,6 +296,22 @@ __device__ __forceinline__ uint64_t add_acquire_sys(uint64_t* p, uint64_t v) {
 }
 __device__ __forceinline__ void red_add_release_sys(uint64_t* p, uint64_t v) {
     asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t cas_acquire_sys(uint64_t* p, uint64_t cmp, uint64_t val) {
+    uint64_t old;
+    asm volatile("atom.acquire.sys.global.cas.b64 %0, [%1], %2, %3;"
+                 : "=l"(old) : "l"(p), "l"(cmp), "l"(val) : "memory");
+    return old;
+}
+/* fault-path PTE RMWs of a region: system scope when a peer cache pins its
+ * pages (dev_region::shared), else GPU scope */
+__device__ __forceinline__ uint64_t pte_cas_acquire(bool shared, uint64_t* p, uint64_t cmp,
+                                                    uint64_t val) {
+    return shared ? cas_acquire_sys(p, cmp, val) : cas_acquire(p, cmp, val);
+}
+__device__ __forceinline__ void pte_red_release(bool shared, uint64_t* p, uint64_t v) {
+    if (shared) red_add_release_sys(p, v);
+    else red_add_release(p, v);
 }
 __device__ __forceinline__ void red_add_relaxed(unsigned long long* p, unsigned long long v) {
     asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -550,7 +571,8 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         /* a dirty victim is claimed into LOADING (faulters wait) until its
          * bytes are back in the file, then released to EMPTY */
         if (elig && __popc(cand & lanemask_lt()) < need_n)
-            won = (cas_acquire(q, e, (e & PTE_DIRTY) ? PTE_LOADING : PTE_EMPTY) == e);
+            won = (pte_cas_acquire(c->regions[(own >> 48) - 1].shared, q, e,
+                                   (e & PTE_DIRTY) ? PTE_LOADING : PTE_EMPTY) == e);
         const unsigned wonm = __ballot_sync(m, won);
         unsigned dirtym = __ballot_sync(m, won && (e & PTE_DIRTY));
         while (dirtym) {
@@ -754,7 +776,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
                 if (!may_claim) {
                     st = ST_SKIP;
                 } else {
-                    const uint64_t prev = cas_acquire(pte, PTE_EMPTY, PTE_LOADING);
+                    const uint64_t prev = pte_cas_acquire(r->shared, pte, PTE_EMPTY, PTE_LOADING);
                     /* prev != 0: transient counts, a racing claimer or a
                      * publish in between; all resolve by retrying */
                     st = prev == PTE_EMPTY ? ST_CLAIMED : ST_WAIT;
@@ -770,7 +792,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame);
             if (st == ST_CLAIMED && !ok) {
                 /* give the page back (an add, so transient counts survive) */
-                red_add_release(pte, (uint64_t)0 - PTE_LOADING);
+                pte_red_release(r->shared, pte, (uint64_t)0 - PTE_LOADING);
                 st = ST_NOFRAME;
             }
         }
@@ -800,9 +822,9 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             if ((int)lane == L) printf("[publish] w%u m%08x n%u f%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, n, f, (unsigned long long)fpg);
 #endif
             if ((int)lane == L)
-                red_add_release(pte, (PTE_VALID - PTE_LOADING) | (AP_REF_ON_FILL ? PTE_REF : 0) |
-                                         ((uint64_t)f << 32) |
-                                         (uint64_t)n);
+                pte_red_release(fr->shared, pte,
+                                (PTE_VALID - PTE_LOADING) | (AP_REF_ON_FILL ? PTE_REF : 0) |
+                                    ((uint64_t)f << 32) | (uint64_t)n);
         }
         const unsigned nminor = __popc(__ballot_sync(m, st == ST_LINKED));
 
@@ -1146,7 +1168,8 @@ struct ptr {
     }
     __device__ __forceinline__ ~ptr() { release(); }
 
-    __device__ __forceinline__ bool linked() const { return (x >> 63) != 0; }
+    /* the valid bit is the sign of the translation's high word: one compare */
+    __device__ __forceinline__ bool linked() const { return (int32_t)(uint32_t)(x >> 32) < 0; }
     /* File offset (xAddress) the pointer designates, linked or not. */
     __device__ __forceinline__ uint64_t foff() const {
         return linked() ? ((page << lg) | (x & ((1ull << lg) - 1))) : x;
@@ -1379,7 +1402,15 @@ struct ptr {
         const uint64_t nb = (uint64_t)(d * (int64_t)sizeof(T));
         step = (int64_t)nb;
         const uint64_t nx = x + nb;
-        const bool cross = linked() && ((x ^ nx) >> lg) != 0;
+        /* A step shorter than the smallest page (4 KiB) leaves the page iff
+         * the page bits of the low word change (a carry into the high word
+         * flips bits lg..31 too, lg <= 21): a 32-bit test.  With a constant
+         * stride the compiler keeps only that branch. */
+        bool cross;
+        if (nb + 4095u < 8191u)
+            cross = linked() && (((uint32_t)x ^ (uint32_t)nx) >> lg) != 0;
+        else
+            cross = linked() && ((x ^ nx) >> lg) != 0;
         const unsigned m = __activemask();
         if (__any_sync(m, cross)) {
             detail::unlink_lanes(m, cross, r, page);

@@ -63,6 +63,7 @@ def _load():
         lib.or_divergent_off.restype = u64
         lib.or_divergent_off.argtypes = [u64, u32, u32, u64, u64, u64]
         lib.or_read_divergent.argtypes = [vp, u64, u32, u32, u64, u32, u64, vp, ci]
+        lib.or_offsets.argtypes = [ci, u64, u32, u32, u64, u64, u32, vp]
         lib.or_block_hist.argtypes = [vp, u32, u32, u64, vp]
         lib.or_floordiv.restype = i64
         lib.or_floordiv.argtypes = [i64, i64]
@@ -131,6 +132,14 @@ def read_divergent(file: np.ndarray, nbytes, page, elem, nthreads, reads, seed, 
     _load().or_read_divergent(_p(file), nbytes, page, elem, nthreads, reads, seed, _p(ck),
                               threads or threads_default())
     return ck
+
+
+def offsets(pattern, nbytes, elem, nthreads, reads, seed, page=0):
+    """uint64[nthreads, reads]: the offset of read i of thread t (pattern
+    1 = UNIFORM over nbytes, 2 = DIVERGENT with pattern page size `page`)."""
+    out = np.empty((nthreads, reads), dtype=np.uint64)
+    _load().or_offsets(pattern, nbytes, page, elem, seed, nthreads, reads, _p(out))
+    return out
 
 
 def perm_idx(k, M):

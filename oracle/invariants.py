@@ -76,6 +76,41 @@ def check(ptes, owner, free_left, frames, require_zero_refcounts=True):
     return errs
 
 
+def link_events(offsets, log2_page, warp=32):
+    """Closed-form number of page links a per-access run performs
+    (Listing 1): `offsets` is
+    uint64[nthreads, reads], the offset each thread reads in access order,
+    threads numbered so that warp w holds threads 32w .. 32w+31.  A thread
+    whose read i lies on the page its read i-1 was on stays linked (no event,
+    PAPER.md:147); every other read needs a link, and at iteration i each
+    distinct page among a warp's needing lanes is linked once, by one leader
+    for the whole group (the count grows by the group size in one step,
+    PAPER.md:157).  So events = sum over (warp, i) of the number of distinct
+    pages among the warp's lanes that left their page (or start, i = 0).
+    With a cache that never runs out of frames each event is exactly one
+    major or one minor fault."""
+    pg = np.asarray(offsets, dtype=np.uint64) >> np.uint64(log2_page)
+    n, reads = pg.shape
+    assert n % warp == 0, "whole warps only"
+    need = np.ones_like(pg, dtype=bool)
+    need[:, 1:] = pg[:, 1:] != pg[:, :-1]
+    key = np.where(need, pg.astype(np.int64), -1)
+    key = key.reshape(n // warp, warp, reads).transpose(0, 2, 1)   # [warp, i, lane]
+    key = np.sort(key, axis=2)
+    distinct = (key[:, :, 1:] != key[:, :, :-1]) & (key[:, :, 1:] >= 0)
+    return int(distinct.sum() + (key[:, :, 0] >= 0).sum())
+
+
+def check_link_count(stats_before, stats_after, expected):
+    """With enough frames (no frame pressure, no eviction) every page link of
+    the run is exactly one major or one minor fault."""
+    got = (stats_after["major"] - stats_before["major"]) + \
+          (stats_after["minor"] - stats_before["minor"])
+    if got != expected:
+        return [f"major+minor = {got} link events, closed form {expected}"]
+    return []
+
+
 def check_fill_counts(stats, distinct_pages, frames, npages_total):
     """Fills happen at least once per distinct page touched, and exactly once
     when the cache can hold every page (no eviction): the LOADING claim

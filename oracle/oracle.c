@@ -140,6 +140,18 @@ void or_read_divergent(const uint8_t* file, uint64_t bytes, uint32_t page, uint3
     }
 }
 
+/* The offsets a random-pattern run reads, in access order: out[t*reads+i]
+ * = the offset of read i of thread t (pattern 1 = UNIFORM over `bytes`,
+ * 2 = DIVERGENT with pattern page size `page`).  Used by the O2 link-count
+ * invariant (oracle/invariants.py link_events). */
+void or_offsets(int pattern, uint64_t bytes, uint32_t page, uint32_t elem, uint64_t seed,
+                uint64_t nthreads, uint32_t reads, uint64_t* out) {
+    for (uint64_t t = 0; t < nthreads; ++t)
+        for (uint32_t i = 0; i < reads; ++i)
+            out[t * reads + i] = pattern == 1 ? or_uniform_off(bytes, elem, seed, t, i)
+                                              : or_divergent_off(bytes, page, elem, seed, t, i);
+}
+
 /* ------------------------------------------------------------------ */
 /* O3 — photo collage                               */
 /* ------------------------------------------------------------------ */

@@ -12,7 +12,9 @@ from . import _lib
 from ._lib import (AP_PROT_READ, AP_PROT_WRITE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_AHEAD, AP_ACCESS_PAIR, AP_ACCESS_TMA, AP_ACCESS_TILE, AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK,  # noqa: F401
                    AP_POLICY_RANDOM, AP_SCHED_LSH, AP_SCHED_NATURAL, AP_SCHED_TABLE, AP_SCHED_TABLE_MH, AP_SEQ,
                    AP_UNIFORM, APError, ap_bench_cfg, ap_collage_in,
-                   ap_stats_t)
+                   ap_stats_t, AP_COLLAGE_ACCUMULATE, AP_COLLAGE_SYSTEM, AP_PART_BLOCKS,
+                   AP_PART_RECORDS, AP_PART_UNITS, AP_MGPU_MAX, ap_ipc_handle_t,
+                   ap_mgpu_collage_in, ap_mgpu_report)
 
 _frames = {}
 
@@ -230,7 +232,7 @@ def ap_bench_latency(cache, region, op, reps=1000):
 def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev, ids_dev, N,
                rec_stride=4096, group=1, block_begin=0, block_count=None,
                mode=AP_MODE_APOINTER, raw_base=None, L=None, K=None, schedule=AP_SCHED_TABLE,
-               unit_begin=0, unit_count=0, id_chunks=0, id_begin=0, id_end=0):
+               unit_begin=0, unit_count=0, id_chunks=0, id_begin=0, id_end=0, flags=0):
     L = proj_dev.shape[0] if L is None else L
     K = proj_dev.shape[1] if K is None else K
     nb = (W // 32) * (H // 32)
@@ -238,12 +240,78 @@ def collage_in(target_dev, W, H, proj_dev, bias_dev, w, bucket_bits, offsets_dev
     return ap_collage_in(_ptr(target_dev), W, H, L, K, bucket_bits, w, _ptr(proj_dev),
                          _ptr(bias_dev), _ptr(offsets_dev), _ptr(ids_dev), N, rec_stride, group,
                          block_begin, block_count, mode, _ptr(raw_base), schedule, unit_begin,
-                         unit_count, id_chunks, id_begin, id_end)
+                         unit_count, id_chunks, id_begin, id_end, flags)
 
 
 def ap_collage_run(cache, region, inp, winners_dev, stream=None):
     _lib.check("ap_collage_run", _lib.lib().ap_collage_run(cache, region, ctypes.byref(inp),
                                                            _ptr(winners_dev), _stream(stream)))
+
+
+def ap_winners_init(winners_dev, nblocks, stream=None):
+    _lib.check("ap_winners_init", _lib.lib().ap_winners_init(_ptr(winners_dev), nblocks,
+                                                             _stream(stream)))
+
+
+def ap_ipc_export(dev_buf):
+    """CUDA IPC handle (ap_ipc_handle_t) of a device buffer of this process."""
+    h = ap_ipc_handle_t()
+    _lib.check("ap_ipc_export", _lib.lib().ap_ipc_export(_ptr(dev_buf), ctypes.byref(h)))
+    return h
+
+
+def ap_ipc_import(handle, device):
+    """Map another process's buffer on `device`; returns its device address."""
+    out = ctypes.c_void_p()
+    _lib.check("ap_ipc_import", _lib.lib().ap_ipc_import(ctypes.byref(handle), device,
+                                                         ctypes.byref(out)))
+    return out.value
+
+
+def ap_ipc_close(dev_ptr):
+    _lib.check("ap_ipc_close", _lib.lib().ap_ipc_close(dev_ptr))
+
+
+def mgpu_collage_in(target_host, W, H, proj_host, bias_host, w, bucket_bits, N, rec_stride=4096,
+                    group=8, schedule=AP_SCHED_TABLE, id_chunks=0, partition=AP_PART_RECORDS):
+    """Host-side inputs of the multi-GPU collage (the arrays must stay alive
+    while the struct is used)."""
+    L, K = bias_host.shape
+    return ap_mgpu_collage_in(_ptr(target_host), W, H, L, K, bucket_bits, w, _ptr(proj_host),
+                              _ptr(bias_host), N, rec_stride, group, schedule, id_chunks,
+                              partition)
+
+
+def ap_mgpu_create(devices, host_file, frames_per_gpu, page_size):
+    devs = (ctypes.c_int * len(devices))(*devices)
+    out = ctypes.c_void_p()
+    _lib.check("ap_mgpu_create", _lib.lib().ap_mgpu_create(
+        len(devices), devs, _ptr(host_file), _nbytes(host_file), frames_per_gpu, page_size,
+        ctypes.byref(out)))
+    return out.value
+
+
+def ap_mgpu_collage(m, inp, winners_host):
+    """One cold step; winners_host = uint32[blocks, 2] host array.  Returns
+    the report as a dict."""
+    rep = ap_mgpu_report()
+    _lib.check("ap_mgpu_collage", _lib.lib().ap_mgpu_collage(m, ctypes.byref(inp),
+                                                             _ptr(winners_host),
+                                                             ctypes.byref(rep)))
+    return rep.as_dict()
+
+
+def ap_mgpu_destroy(m):
+    _lib.check("ap_mgpu_destroy", _lib.lib().ap_mgpu_destroy(m))
+
+
+def ap_collage_mgpu(devices, host_file, frames_per_gpu, page_size, inp, winners_host):
+    devs = (ctypes.c_int * len(devices))(*devices)
+    rep = ap_mgpu_report()
+    _lib.check("ap_collage_mgpu", _lib.lib().ap_collage_mgpu(
+        len(devices), devs, _ptr(host_file), _nbytes(host_file), frames_per_gpu, page_size,
+        ctypes.byref(inp), _ptr(winners_host), ctypes.byref(rep)))
+    return rep.as_dict()
 
 
 def ap_lsh_build_index(cache, region, N, rec_stride, L, K, bucket_bits, w, proj_dev, bias_dev,

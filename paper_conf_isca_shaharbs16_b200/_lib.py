@@ -50,7 +50,36 @@ class ap_collage_in(ctypes.Structure):
                 ("offsets_dev", vp), ("ids_dev", vp), ("N", u64), ("rec_stride", u32),
                 ("group", u32), ("block_begin", u64), ("block_count", u64), ("mode", i32),
                 ("raw_base", vp), ("schedule", i32), ("unit_begin", u64), ("unit_count", u64),
-                ("id_chunks", u32), ("id_begin", u32), ("id_end", u32)]
+                ("id_chunks", u32), ("id_begin", u32), ("id_end", u32), ("flags", u32)]
+
+
+AP_COLLAGE_ACCUMULATE, AP_COLLAGE_SYSTEM = 1, 2
+AP_PART_BLOCKS, AP_PART_RECORDS, AP_PART_UNITS = 0, 1, 2
+AP_MGPU_MAX = 16
+
+
+class ap_ipc_handle_t(ctypes.Structure):
+    _fields_ = [("handle", ctypes.c_uint8 * 64), ("offset", u64), ("bytes", u64),
+                ("device", i32), ("pid", i32)]
+
+
+class ap_mgpu_collage_in(ctypes.Structure):
+    _fields_ = [("target_host", vp), ("W", u32), ("H", u32), ("L", u32), ("K", u32),
+                ("bucket_bits", u32), ("w", i32), ("proj_host", vp), ("bias_host", vp),
+                ("N", u64), ("rec_stride", u32), ("group", u32), ("schedule", i32),
+                ("id_chunks", u32), ("partition", i32)]
+
+
+class ap_mgpu_report(ctypes.Structure):
+    _fields_ = [("seconds", ctypes.c_double), ("part_seconds", ctypes.c_double * AP_MGPU_MAX),
+                ("fill_bytes", u64 * AP_MGPU_MAX), ("major", u64 * AP_MGPU_MAX),
+                ("device_error", i32), ("nparts", i32)]
+
+    def as_dict(self):
+        n = self.nparts
+        return {"seconds": self.seconds, "part_seconds": list(self.part_seconds[:n]),
+                "fill_bytes": [int(x) for x in self.fill_bytes[:n]],
+                "major": [int(x) for x in self.major[:n]], "device_error": self.device_error}
 
 
 class ap_compute_cfg(ctypes.Structure):
@@ -109,6 +138,18 @@ def lib():
             "ap_region_clear_peers": (ci, [vp, u32]),
             "ap_lsh_build_index": (ci, [vp, u32, u64, u32, u32, u32, u32, i32, vp, vp, vp, vp,
                                         vp]),
+            "ap_winners_init": (ci, [vp, u64, vp]),
+            "ap_ipc_export": (ci, [vp, ctypes.POINTER(ap_ipc_handle_t)]),
+            "ap_ipc_import": (ci, [ctypes.POINTER(ap_ipc_handle_t), ci, ctypes.POINTER(vp)]),
+            "ap_ipc_close": (ci, [vp]),
+            "ap_mgpu_create": (ci, [ci, ctypes.POINTER(ci), vp, u64, u64, u32,
+                                    ctypes.POINTER(vp)]),
+            "ap_mgpu_collage": (ci, [vp, ctypes.POINTER(ap_mgpu_collage_in), vp,
+                                     ctypes.POINTER(ap_mgpu_report)]),
+            "ap_mgpu_destroy": (ci, [vp]),
+            "ap_collage_mgpu": (ci, [ci, ctypes.POINTER(ci), vp, u64, u64, u32,
+                                     ctypes.POINTER(ap_mgpu_collage_in), vp,
+                                     ctypes.POINTER(ap_mgpu_report)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -125,7 +166,9 @@ EXPORTED = ["ap_strerror", "ap_version", "ap_cache_create", "ap_cache_destroy", 
             "ap_bench_read", "ap_bench_read_host", "ap_collage_run", "ap_lsh_build_index",
             "ap_bench_latency", "ap_mmap_prot", "ap_msync", "ap_bench_write", "ap_bench_copy",
             "ap_bench_compute", "ap_cache_set_backoff", "ap_region_add_peer", "ap_region_export",
-            "ap_region_add_peer_ipc", "ap_region_clear_peers"]
+            "ap_region_add_peer_ipc", "ap_region_clear_peers", "ap_winners_init",
+            "ap_ipc_export", "ap_ipc_import", "ap_ipc_close", "ap_mgpu_create",
+            "ap_mgpu_collage", "ap_mgpu_destroy", "ap_collage_mgpu"]
 
 
 def check(fn, rc):

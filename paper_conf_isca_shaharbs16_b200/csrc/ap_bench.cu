@@ -17,6 +17,8 @@
  */
 #include <cuda_runtime.h>
 
+#include <algorithm>
+
 #include "ap_internal.cuh"
 
 /* The apointer kernels need ~120 registers once the fault path is linked
@@ -93,6 +95,13 @@ __device__ __forceinline__ void consume(const BenchArgs& a, uint64_t off, const 
     if (a.out_copy) *reinterpret_cast<T*>(a.out_copy + off) = v;
     else h = fnv(h, v);
 }
+/* the same with the output kind fixed at compile time (per-access loops) */
+template <bool COPY, class T>
+__device__ __forceinline__ void consume_k(const BenchArgs& a, uint64_t off, const T& v,
+                                          uint64_t& h) {
+    if constexpr (COPY) *reinterpret_cast<T*>(a.out_copy + off) = v;
+    else h = fnv(h, v);
+}
 
 /* raw-pointer reader with the apointer's interface (the twin) */
 template <class T>
@@ -139,27 +148,67 @@ __device__ __forceinline__ void seq_unit(R& q, const BenchArgs& a, uint64_t e0, 
     }
 }
 
-/* one unit, one access at a time: `v = *q; q += 32` (the paper's loop) */
-template <class T>
-__device__ __forceinline__ void seq_unit_deref(ap::ptr<T>& q, const BenchArgs& a, uint64_t e0,
-                                               uint32_t per_unit, uint64_t& h) {
+/* One unit, one access at a time: `v = *q; q += 32` (the paper's loop,
+ * PAPER.md:310-316, 336), the same source for the apointer and its raw twin.
+ *
+ * Every access is its own dereference (its own translation check, its own
+ * possible fault), so the only way for a warp to keep more than one load in
+ * flight is to issue access j+D before it consumes access j: the loop keeps
+ * the last D values in registers (AP_DEREF_PIPE; the pointer moves on before
+ * the value it produced is used).  A check or a fault of access j+D then
+ * never waits for the data of access j, and no loaded value is live across
+ * the out-of-line fault path of the access that issues it (deref_slow reloads
+ * lanes that were linked).  D = 1 is the plain loop. */
+#ifndef AP_DEREF_PIPE
+#define AP_DEREF_PIPE 4
+#endif
+template <class T, bool COPY, class R>
+__device__ __forceinline__ void seq_unit_deref(R& q, const BenchArgs& a, uint64_t e0,
+                                               uint32_t per_unit, bool whole, uint64_t& h) {
     constexpr uint32_t E = sizeof(T);
-    for (uint32_t j = 0; j < per_unit; ++j) {
+    constexpr int D = AP_DEREF_PIPE;
+    uint32_t j = 0;
+    if (D > 1 && whole && per_unit >= (uint32_t)D) {
+        T v[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) {
+            v[d] = *q;
+            q += 32;
+        }
+        /* the ring holds accesses j .. j+D-1 */
+        for (; j + 2 * D <= per_unit; j += D) {
+#pragma unroll
+            for (int d = 0; d < D; ++d) {
+                const T nv = *q; /* access j + d + D */
+                q += 32;
+                consume_k<COPY>(a, (e0 + 32ull * (j + d)) * E, v[d], h);
+                v[d] = nv;
+            }
+        }
+#pragma unroll
+        for (int d = 0; d < D; ++d) consume_k<COPY>(a, (e0 + 32ull * (j + d)) * E, v[d], h);
+        j += D; /* per_unit % D accesses remain for the loop below */
+    }
+    for (; j < per_unit; ++j) {
         const uint64_t off = (e0 + 32ull * j) * E;
-        if (off + E <= a.span) consume(a, off, (T)*q, h);
-        q += 32;
+        if (off + E <= a.span) {
+            const T v = *q;
+            q += 32;
+            consume_k<COPY>(a, off, v, h);
+        } else {
+            q += 32;
+        }
     }
 }
 
-/* The per-access form keeps one load in flight per warp (each access may
- * enter the fault path), so it needs warps, not registers: this kernel is
- * built for AP_DEREF_MINB CTAs of 512 threads per SM (full occupancy at 4,
- * 32 registers; the out-of-line fault path spills, the hit path does not).
- * The raw twin runs the same per-access loop on a plain pointer. */
+/* The per-access form needs loads in flight more than registers: built for
+ * AP_DEREF_MINB CTAs of 512 threads per SM (2 = 64 registers, the paper's
+ * register budget).  The raw twin runs the identical loop on a
+ * plain pointer at the same launch. */
 #ifndef AP_DEREF_MINB
-#define AP_DEREF_MINB 4
+#define AP_DEREF_MINB 2
 #endif
-template <class T, bool APTR>
+template <class T, bool APTR, bool COPY>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_DEREF_MINB)
     k_seq_deref(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
     constexpr uint32_t E = sizeof(T);
@@ -172,20 +221,17 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_DEREF_MINB)
     for (uint32_t pass = 0; pass < a.passes; ++pass) {
         for (uint64_t u = w; u < nunits; u += W) {
             const uint64_t e0 = u * (a.unit / E) + lane;
+            const bool whole = (u + 1) * a.unit <= a.span;
             if constexpr (APTR) {
                 ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
-                seq_unit_deref<T>(q, a, e0, per_unit, h);
+                seq_unit_deref<T, COPY>(q, a, e0, per_unit, whole, h);
             } else {
                 raw_reader<T> q{reinterpret_cast<const T*>(a.raw) + e0};
-                for (uint32_t j = 0; j < per_unit; ++j) {
-                    const uint64_t off = (e0 + 32ull * j) * E;
-                    if (off + E <= a.span) consume(a, off, *q, h);
-                    q += 32;
-                }
+                seq_unit_deref<T, COPY>(q, a, e0, per_unit, whole, h);
             }
         }
     }
-    if (!a.out_copy) a.ck[t] = h;
+    if constexpr (!COPY) a.ck[t] = h;
 }
 
 /* AP_ACCESS_AHEAD: the tiled loop with a split-phase link.  The warp's next
@@ -379,7 +425,10 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, 1)
             if constexpr (APTR) {
                 q[k & 1] = ap::gvmmap<uint4>(c, region, u * a.unit);
                 const uint4* p = q[k & 1].pin_range(a.unit);
-                ubase[k & 1] = reinterpret_cast<const uint8_t*>(p);
+                /* a failed pin (the fault path's watchdog; make_args rules out
+                 * frame exhaustion) has set the sticky error: copy from the
+                 * frame pool, always mapped, instead of address 0 */
+                ubase[k & 1] = p ? reinterpret_cast<const uint8_t*>(p) : c->pool;
                 /* frame data written by the generic proxy (fills), read by
                  * the async proxy (TMA) */
                 asm volatile("fence.proxy.async.global;" ::: "memory");
@@ -452,8 +501,12 @@ cudaError_t launch_t(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg
                      const BenchArgs& a, cudaStream_t s) {
     switch (cfg->pattern) {
         case AP_SEQ:
-            if (cfg->access == AP_ACCESS_DEREF)
-                k_seq_deref<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            if (cfg->access == AP_ACCESS_DEREF) {
+                if (a.out_copy)
+                    k_seq_deref<T, APTR, true><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+                else
+                    k_seq_deref<T, APTR, false><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            }
             else if (APTR && (cfg->access == AP_ACCESS_AHEAD || cfg->access == AP_ACCESS_PAIR))
                 k_seq_split<T><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             else if (cfg->access == AP_ACCESS_TMA) {
@@ -515,9 +568,14 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
             else a->ck = (uint64_t*)out;
             /* TMA staging: 16-B checksums over whole units of whole stages,
              * at least as many stages per unit as are in flight */
+            /* each warp pins up to two units at once (the next unit's pin
+             * overlaps the current unit's stages): frames >= 2 per resident
+             * warp, so no warp ever waits for a frame while pinning one */
             if (cfg->access == AP_ACCESS_TMA &&
                 (E != 16 || cfg->out_copy || a->unit % TMA_SB || a->unit / TMA_SB < TMA_ST ||
-                 a->span % a->unit || cfg->block > AP_BENCH_THREADS))
+                 a->span % a->unit || cfg->block > AP_BENCH_THREADS ||
+                 (cfg->mode == AP_MODE_APOINTER && c->frames < rg.npages &&
+                  c->frames < 2ull * std::min<uint64_t>(cfg->grid, c->num_sms) * (cfg->block / 32))))
                 return AP_EINVAL;
             break;
         case AP_UNIFORM: /* offsets uniform over [0, span) (span 0 = the region) */

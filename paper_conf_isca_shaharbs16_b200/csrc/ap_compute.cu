@@ -120,12 +120,85 @@ __device__ __forceinline__ unsigned long long work_elem(const uint4& v, const ui
            work_word<WORK>(v.z, v2.z, lane, iters) + work_word<WORK>(v.w, v2.w, lane, iters);
 }
 
-/* per-access loops need warps, not registers: built for full occupancy
- * (4 CTAs of 512 threads per SM, 32 registers), the sweep's upper end as in
- * the paper's Fig. 6 x axis */
+/* Per-access loops keep up to AP_COMPUTE_PIPE accesses in flight per lane:
+ * access j + D is dereferenced (and its pointer moved on) before the value of
+ * access j is used, so no check or fault of a later access waits for an
+ * earlier access's data (the same source for both pointer types).  Built
+ * for AP_COMPUTE_MINB CTAs of 512 threads per SM (2 = 64 registers, the
+ * paper's budget). */
 #ifndef AP_COMPUTE_MINB
-#define AP_COMPUTE_MINB 1
+#define AP_COMPUTE_MINB 2
 #endif
+#ifndef AP_COMPUTE_PIPE
+#define AP_COMPUTE_PIPE 4
+#endif
+/* ADD keeps two values per access in the ring */
+#ifndef AP_COMPUTE_PIPE_ADD
+#define AP_COMPUTE_PIPE_ADD (AP_COMPUTE_PIPE > 1 ? AP_COMPUTE_PIPE / 2 : 1)
+#endif
+
+/* one access of the Fig. 6 loop through apointers: `v = *q` (and `v2 = *q2`
+ * for ADD), then both pointers move on */
+template <class T, int WORK>
+struct ap_access {
+    ap::ptr<T> q, q2;
+    __device__ __forceinline__ void next(T& v, T& v2) {
+        /* ADD holds two pointers: never fault one while the other pins a
+         * frame of a recycled cache (R-A19) */
+        if (WORK == 0 && !q.linked_all() && q.cache_pressure()) q2.release();
+        v = *q;
+        q += 32;
+        if (WORK == 0) {
+            if (!q2.linked_all() && q2.cache_pressure()) q.release();
+            v2 = *q2;
+            q2 += 32;
+        }
+    }
+};
+template <class T, int WORK>
+struct raw_access {
+    const T* q;
+    int64_t second;
+    __device__ __forceinline__ void next(T& v, T& v2) {
+        v = ap::detail::ld_data<T>(q);
+        if (WORK == 0) v2 = ap::detail::ld_data<T>(q + second);
+        q += 32;
+    }
+};
+
+template <class T, int WORK, class A>
+__device__ __forceinline__ void compute_unit(A& acc_ptr, uint32_t per_unit, unsigned lane,
+                                             uint32_t iters, unsigned long long& acc) {
+    constexpr int D = WORK == 0 ? AP_COMPUTE_PIPE_ADD : AP_COMPUTE_PIPE;
+    uint32_t j = 0;
+    if (D > 1 && per_unit >= (uint32_t)D) {
+        T v[D], v2[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) {
+            v2[d] = T{};
+            acc_ptr.next(v[d], v2[d]);
+        }
+        for (; j + 2 * D <= per_unit; j += D) {
+#pragma unroll
+            for (int d = 0; d < D; ++d) {
+                T nv, nv2{};
+                acc_ptr.next(nv, nv2);
+                acc += work_elem<WORK>(v[d], v2[d], lane, iters);
+                v[d] = nv;
+                v2[d] = nv2;
+            }
+        }
+#pragma unroll
+        for (int d = 0; d < D; ++d) acc += work_elem<WORK>(v[d], v2[d], lane, iters);
+        j += D;
+    }
+    for (; j < per_unit; ++j) {
+        T v, v2{};
+        acc_ptr.next(v, v2);
+        acc += work_elem<WORK>(v, v2, lane, iters);
+    }
+}
+
 template <class T, int WORK, bool APTR>
 __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_COMPUTE_MINB)
     k_compute(const ap::dev_cache* __restrict__ c, uint32_t region, const CompArgs a) {
@@ -141,32 +214,13 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_COMPUTE_MINB)
     for (uint64_t u = w; u < nunits; u += W) {
         const uint64_t e0 = u * (a.unit / E) + lane;
         if constexpr (APTR) {
-            ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
-            [[maybe_unused]] ap::ptr<T> q2;
-            if (WORK == 0) q2 = ap::gvmmap<T>(c, region, (e0 + second) * E);
-            for (uint32_t j = 0; j < per_unit; ++j) {
-                /* ADD holds two pointers: never fault one while the other
-                 * pins a frame of a recycled cache (R-A19) */
-                if (WORK == 0 && !q.linked_all() && q.cache_pressure()) q2.release();
-                const T v = *q;
-                T v2{};
-                if (WORK == 0) {
-                    if (!q2.linked_all() && q2.cache_pressure()) q.release();
-                    v2 = *q2;
-                    q2 += 32;
-                }
-                acc += work_elem<WORK>(v, v2, lane, a.iters);
-                q += 32;
-            }
+            ap_access<T, WORK> p;
+            p.q = ap::gvmmap<T>(c, region, e0 * E);
+            if (WORK == 0) p.q2 = ap::gvmmap<T>(c, region, (e0 + second) * E);
+            compute_unit<T, WORK>(p, per_unit, lane, a.iters, acc);
         } else {
-            const T* q = reinterpret_cast<const T*>(a.raw) + e0;
-            for (uint32_t j = 0; j < per_unit; ++j) {
-                const T v = ap::detail::ld_data<T>(q);
-                T v2{};
-                if (WORK == 0) v2 = ap::detail::ld_data<T>(q + second);
-                acc += work_elem<WORK>(v, v2, lane, a.iters);
-                q += 32;
-            }
+            raw_access<T, WORK> p{reinterpret_cast<const T*>(a.raw) + e0, second};
+            compute_unit<T, WORK>(p, per_unit, lane, a.iters, acc);
         }
     }
     a.out[t] = acc;

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <utility>
 #include <vector>
 
 #include "ap.h"
@@ -19,12 +20,19 @@ struct ap_region_host {
     uint64_t bytes = 0;
     uint64_t npages = 0;
     uint64_t* pte = nullptr; /* device                                     */
-    bool registered = false; /* we called cudaHostRegister                 */
+    const void* reg_base = nullptr; /* the library's host registration this
+                                     * region holds a reference on, or null  */
     bool live = false;
     uint32_t prot = 1;       /* AP_PROT_*                                  */
     std::vector<ap::dev_peer> peers;  /* N2 peer caches (device-readable)  */
     ap::dev_peer* d_peers = nullptr;  /* their device copy                 */
     std::vector<void*> ipc_opened;    /* CUDA IPC mappings to close        */
+    /* same-process peers: the regions this region copies from, and the
+     * regions that copy from this one (its page table and frames must stay
+     * alive while they do: ap_munmap answers AP_EBUSY) */
+    std::vector<std::pair<struct ap_cache_s*, ap_region_t>> peer_src;
+    std::vector<std::pair<struct ap_cache_s*, ap_region_t>> importers;
+    bool exported = false; /* handed out with ap_region_export */
 };
 
 struct ap_cache_s {

@@ -4,12 +4,14 @@
  * statistics, reset, dumps, prefill.  C ABI in include/ap.h.
  */
 #include <cuda_runtime.h>
+#include <cstddef>
 #include <cstring>
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
+#include <mutex>
 #include <vector>
 
 #include "ap_internal.cuh"
@@ -291,6 +293,41 @@ extern "C" int ap_cache_destroy(ap_cache_t c) {
 }
 
 /* ------------------------------------------------------------ regions */
+/* Host registrations the library made, shared by every cache of the process
+ * (several caches -- one per GPU -- map the same file): a registration is
+ * undone only when the last region using it is unmapped.  Registrations the
+ * caller made (cudaHostRegister / cudaHostAlloc / torch pin_memory) are used
+ * as they are and never undone here. */
+namespace {
+struct host_reg {
+    const uint8_t* base;
+    uint64_t bytes;
+    int refs;
+    bool readonly;
+};
+std::mutex g_reg_mu;
+std::vector<host_reg> g_regs;
+
+host_reg* find_reg(const void* p, uint64_t bytes) {
+    const uint8_t* b = (const uint8_t*)p;
+    for (auto& r : g_regs)
+        if (b >= r.base && b + bytes <= r.base + r.bytes) return &r;
+    return nullptr;
+}
+}  // namespace
+
+static void release_host_reg(const void* base) {
+    std::lock_guard<std::mutex> lk(g_reg_mu);
+    for (size_t i = 0; i < g_regs.size(); ++i)
+        if (g_regs[i].base == (const uint8_t*)base) {
+            if (--g_regs[i].refs == 0) {
+                cudaHostUnregister(const_cast<uint8_t*>(g_regs[i].base));
+                cudaGetLastError();
+                g_regs.erase(g_regs.begin() + i);
+            }
+            return;
+        }
+}
 extern "C" int ap_mmap(ap_cache_t c, const void* host_buf, uint64_t bytes, ap_region_t* out) {
     return ap_mmap_prot(c, host_buf, bytes, AP_PROT_READ, out);
 }
@@ -313,74 +350,112 @@ extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, 
     rg.host_buf = host_buf;
     rg.bytes = bytes;
     rg.npages = npages;
-    cudaPointerAttributes attr{};
-    cudaError_t e = cudaPointerGetAttributes(&attr, host_buf);
-    cudaGetLastError();
-    if (e == cudaSuccess && attr.type == cudaMemoryTypeHost && attr.devicePointer) {
-        rg.dev_alias = (const uint8_t*)attr.devicePointer;
-    } else if (e == cudaSuccess && attr.type == cudaMemoryTypeDevice) {
-        return AP_EINVAL; /* the backing store is host memory */
-    } else {
-        unsigned flags = cudaHostRegisterMapped | cudaHostRegisterPortable;
-        int ro = 0;
-        if (!(prot & AP_PROT_WRITE))
-            cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->device);
-        if (ro) flags |= cudaHostRegisterReadOnly;
-        e = cudaHostRegister(const_cast<void*>(host_buf), bytes, flags);
-        if (e != cudaSuccess && ro) {
-            cudaGetLastError();
-            e = cudaHostRegister(const_cast<void*>(host_buf), bytes,
-                                 cudaHostRegisterMapped | cudaHostRegisterPortable);
+    {
+        std::lock_guard<std::mutex> lk(g_reg_mu);
+        host_reg* hr = find_reg(host_buf, bytes);
+        if (hr) {
+            /* a registration this library made for another region/cache:
+             * share it (a writable mapping cannot use a read-only one) */
+            if ((prot & AP_PROT_WRITE) && hr->readonly) return AP_EINVAL;
+            void* dp = nullptr;
+            if (cudaHostGetDevicePointer(&dp, const_cast<void*>(host_buf), 0) != cudaSuccess) {
+                cudaGetLastError();
+                return AP_ECUDA;
+            }
+            rg.dev_alias = (const uint8_t*)dp;
+            rg.reg_base = hr->base;
+            ++hr->refs;
         }
-        if (e != cudaSuccess) {
-            cudaGetLastError();
-            return AP_ENOMEM;
-        }
-        rg.registered = true;
-        void* dp = nullptr;
-        if (cudaHostGetDevicePointer(&dp, const_cast<void*>(host_buf), 0) != cudaSuccess) {
-            cudaHostUnregister(const_cast<void*>(host_buf));
-            return AP_ECUDA;
-        }
-        rg.dev_alias = (const uint8_t*)dp;
     }
-    if (cudaMalloc(&rg.pte, npages * 8) != cudaSuccess) {
-        if (rg.registered) cudaHostUnregister(const_cast<void*>(host_buf));
+    if (!rg.dev_alias) {
+        cudaPointerAttributes attr{};
+        cudaError_t e = cudaPointerGetAttributes(&attr, host_buf);
         cudaGetLastError();
-        return AP_ENOMEM;
+        if (e == cudaSuccess && attr.type == cudaMemoryTypeHost && attr.devicePointer) {
+            /* pinned and mapped by the caller: used as is, never unregistered */
+            rg.dev_alias = (const uint8_t*)attr.devicePointer;
+        } else if (e == cudaSuccess && attr.type == cudaMemoryTypeDevice) {
+            return AP_EINVAL; /* the backing store is host memory */
+        } else {
+            unsigned flags = cudaHostRegisterMapped | cudaHostRegisterPortable;
+            int ro = 0;
+            if (!(prot & AP_PROT_WRITE))
+                cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->device);
+            if (ro) flags |= cudaHostRegisterReadOnly;
+            e = cudaHostRegister(const_cast<void*>(host_buf), bytes, flags);
+            if (e != cudaSuccess && ro) {
+                cudaGetLastError();
+                ro = 0;
+                e = cudaHostRegister(const_cast<void*>(host_buf), bytes,
+                                     cudaHostRegisterMapped | cudaHostRegisterPortable);
+            }
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                return AP_ENOMEM;
+            }
+            void* dp = nullptr;
+            if (cudaHostGetDevicePointer(&dp, const_cast<void*>(host_buf), 0) != cudaSuccess) {
+                cudaHostUnregister(const_cast<void*>(host_buf));
+                cudaGetLastError();
+                return AP_ECUDA;
+            }
+            rg.dev_alias = (const uint8_t*)dp;
+            rg.reg_base = host_buf;
+            std::lock_guard<std::mutex> lk(g_reg_mu);
+            g_regs.push_back(host_reg{(const uint8_t*)host_buf, bytes, 1, ro != 0});
+        }
     }
-    AP_CUDA_TRY(cudaMemset(rg.pte, 0, npages * 8));
+    /* every failure below releases the registration reference taken above */
+    auto fail = [&](int code) {
+        if (rg.pte) cudaFree(rg.pte);
+        if (rg.reg_base) release_host_reg(rg.reg_base);
+        cudaGetLastError();
+        return code;
+    };
+    if (cudaMalloc(&rg.pte, npages * 8) != cudaSuccess) {
+        rg.pte = nullptr;
+        return fail(AP_ENOMEM);
+    }
+    if (cudaMemset(rg.pte, 0, npages * 8) != cudaSuccess) return fail(AP_ECUDA);
 #ifdef AP_PT_HASH
     if (2 * (c->slot_keys + npages) > (1ull << c->slot_bits)) {
         /* grow the table to >= 2x the keys: dirty pages go back to their
-         * files first, then every page is evicted (a reset) */
+         * files, every page is evicted (a reset, which checks the live
+         * table for references first), then the regions move to a fresh
+         * table; the old keys and tombstones are gone, so the key count
+         * restarts from the mapped pages */
         for (uint32_t i = 0; i < c->reg.size(); ++i)
             if (c->reg[i].live && (c->reg[i].prot & AP_PROT_WRITE)) {
                 int rcw = ap_msync(c, i);
-                if (rcw) return rcw;
+                if (rcw) return fail(rcw);
             }
+        int rcr = ap_cache_reset(c);
+        if (rcr) return fail(rcr);
+        uint64_t live_pages = 0;
+        for (uint32_t i = 0; i < c->reg.size(); ++i)
+            if (c->reg[i].live) live_pages += c->reg[i].npages;
         uint32_t bits = c->slot_bits;
-        while ((1ull << bits) < 2 * (c->slot_keys + npages)) ++bits;
+        while ((1ull << bits) < 2 * (live_pages + npages)) ++bits;
         uint64_t* ns = nullptr;
-        if (cudaMalloc(&ns, 16ull << bits) != cudaSuccess) {
-            cudaGetLastError();
-            return AP_ENOMEM;
+        if (cudaMalloc(&ns, 16ull << bits) != cudaSuccess) return fail(AP_ENOMEM);
+        if (cudaMemset(ns, 0, 16ull << bits) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
+            cudaFree(ns);
+            return fail(AP_ECUDA);
         }
-        AP_CUDA_TRY(cudaMemset(ns, 0, 16ull << bits));
-        AP_CUDA_TRY(cudaDeviceSynchronize());
         cudaFree(c->slots);
         c->slots = ns;
         c->slot_bits = bits;
         for (uint32_t i = 0; i < c->reg.size(); ++i)
             if (c->reg[i].live) {
                 ap::dev_region od{};
-                AP_CUDA_TRY(cudaMemcpy(&od, c->regions + i, sizeof od, cudaMemcpyDeviceToHost));
+                if (cudaMemcpy(&od, c->regions + i, sizeof od, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    return fail(AP_ECUDA);
                 od.pte = c->slots;
                 od.pad_ = c->slot_bits;
-                AP_CUDA_TRY(cudaMemcpy(c->regions + i, &od, sizeof od, cudaMemcpyHostToDevice));
+                if (cudaMemcpy(c->regions + i, &od, sizeof od, cudaMemcpyHostToDevice) != cudaSuccess)
+                    return fail(AP_ECUDA);
             }
-        int rcr = ap_cache_reset(c);
-        if (rcr) return rcr;
+        c->slot_keys = live_pages;
     }
     c->slot_keys += npages;
 #endif
@@ -400,7 +475,8 @@ extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, 
     d.prot = (uint32_t)prot;
     d.id = id;
     d.live = 1;
-    AP_CUDA_TRY(cudaMemcpy(c->regions + id, &d, sizeof d, cudaMemcpyHostToDevice));
+    if (cudaMemcpy(c->regions + id, &d, sizeof d, cudaMemcpyHostToDevice) != cudaSuccess)
+        return fail(AP_ECUDA);
     rg.live = true;
     rg.prot = (uint32_t)prot;
     if (id == c->reg.size()) c->reg.push_back(rg);
@@ -422,6 +498,9 @@ extern "C" int ap_msync(ap_cache_t c, ap_region_t r) {
 
 extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
     if (!ap_region_ok(c, r)) return AP_EINVAL;
+    /* another cache still copies from this region's frames (a same-process
+     * peer, ap_region_add_peer): it must clear its peers first */
+    if (!c->reg[r].importers.empty()) return AP_EBUSY;
     ap_device_guard g(c->device);
     AP_CUDA_TRY(cudaDeviceSynchronize());
     if (!c->reg[r].peers.empty() || c->reg[r].d_peers) {
@@ -449,12 +528,22 @@ extern "C" int ap_munmap(ap_cache_t c, ap_region_t r) {
     AP_CUDA_TRY(cudaMemset(c->regions + r, 0, sizeof(ap::dev_region)));
     AP_CUDA_TRY(cudaDeviceSynchronize());
     cudaFree(rg.pte);
-    if (rg.registered) cudaHostUnregister(const_cast<void*>(rg.host_buf));
+    if (rg.reg_base) release_host_reg(rg.reg_base);
     rg = ap_region_host{};
     return AP_OK;
 }
 
 /* ------------------------------------------------------------ N2 peers */
+/* dev_region::shared: the fault path's claim / publish / eviction RMWs on
+ * this region's PTEs use system scope once another cache pins its pages */
+static int set_region_shared(ap_cache_s* c, ap_region_t r, uint32_t v) {
+    ap_device_guard g(c->device);
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    AP_CUDA_TRY(cudaMemcpy((uint8_t*)(c->regions + r) + offsetof(ap::dev_region, shared), &v,
+                           sizeof v, cudaMemcpyHostToDevice));
+    return AP_OK;
+}
+
 static int push_region_peers(ap_cache_s* c, ap_region_t r) {
     ap_region_host& rg = c->reg[r];
     if (!rg.d_peers && cudaMalloc(&rg.d_peers, sizeof(ap::dev_peer) * ap::MAX_PEERS) != cudaSuccess) {
@@ -499,8 +588,19 @@ extern "C" int ap_region_add_peer(ap_cache_t c, ap_region_t r, ap_cache_t pc, ap
         else AP_CUDA_TRY(e);
     }
     AP_CUDA_TRY(cudaDeviceSynchronize());
+    if (pc->reg[pr].importers.empty() && !pc->reg[pr].exported) {
+        rc = set_region_shared(pc, pr, 1);
+        if (rc) return rc;
+    }
     c->reg[r].peers.push_back(ap::dev_peer{pc->reg[pr].pte, pc->pool});
-    return push_region_peers(c, r);
+    rc = push_region_peers(c, r);
+    if (rc) {
+        c->reg[r].peers.pop_back();
+        return rc;
+    }
+    c->reg[r].peer_src.emplace_back(pc, pr);
+    pc->reg[pr].importers.emplace_back(c, r);
+    return AP_OK;
 }
 
 extern "C" int ap_region_export(ap_cache_t c, ap_region_t r, ap_peer_handle_t* out) {
@@ -521,6 +621,11 @@ extern "C" int ap_region_export(ap_cache_t c, ap_region_t r, ap_peer_handle_t* o
     h.bytes = c->reg[r].bytes;
     h.page_size = c->page;
     h.device = c->device;
+    if (!c->reg[r].exported && c->reg[r].importers.empty()) {
+        int rc = set_region_shared(c, r, 1);
+        if (rc) return rc;
+    }
+    c->reg[r].exported = true;
     *out = h;
     return AP_OK;
 }
@@ -563,6 +668,16 @@ extern "C" int ap_region_clear_peers(ap_cache_t c, ap_region_t r) {
     }
     for (void* p : rg.ipc_opened) cudaIpcCloseMemHandle(p);
     rg.ipc_opened.clear();
+    /* the same-process peers no longer have this importer */
+    for (auto& src : rg.peer_src) {
+        auto& imp = src.first->reg[src.second].importers;
+        for (size_t i = 0; i < imp.size(); ++i)
+            if (imp[i].first == c && imp[i].second == r) {
+                imp.erase(imp.begin() + i);
+                break;
+            }
+    }
+    rg.peer_src.clear();
     return AP_OK;
 }
 
@@ -605,6 +720,13 @@ extern "C" int ap_cache_stats(ap_cache_t c, ap_stats_t* out) {
 
 extern "C" int ap_cache_reset(ap_cache_t c) {
     if (!c) return AP_EINVAL;
+    /* caches that copy from this one (same-process peers) may have kernels
+     * in flight on other GPUs pinning our frames: let them finish first */
+    for (auto& rg : c->reg)
+        for (auto& imp : rg.importers) {
+            ap_device_guard gi(imp.first->device);
+            AP_CUDA_TRY(cudaDeviceSynchronize());
+        }
     ap_device_guard g(c->device);
     AP_CUDA_TRY(cudaDeviceSynchronize());
     for (auto& rg : c->reg) {

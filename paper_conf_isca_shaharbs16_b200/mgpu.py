@@ -15,7 +15,19 @@
   the file and every record is filled by exactly one rank (a data-parallel
   split of the file itself); winners are MIN-reduced like the bucket split.
 
-NCCL over NVLink on GPUs; gloo in the CPU tests.  Marshalling only.
+Two ways to combine the winners:
+
+* fused (SharedWinners, the default): rank 0's winners array is mapped into
+  every rank's process with CUDA IPC (ap_ipc_export / ap_ipc_import) and each
+  rank's collage kernel folds its blocks' results straight into it with a
+  system-scope 64-bit atomic min over NVLink (ap_collage_in.flags =
+  AP_COLLAGE_ACCUMULATE | AP_COLLAGE_SYSTEM): no collective in the data path,
+  the combine overlaps the other ranks' kernels.  The arithmetic is in the
+  kernel; this module only exchanges the IPC handle and synchronises.
+* NCCL (gather_winners / reduce_winners_min): one gather or one MIN reduce
+  over torch.distributed, the baseline the fused path replaces.
+
+gloo in the CPU tests.  Marshalling only.
 """
 
 
@@ -74,3 +86,56 @@ def reduce_winners_min(win, rank, world, dist, dst=0):
     if rank != dst:
         return None
     return (w64 ^ flip).view(torch.int32).view(-1, 2)
+
+
+class SharedWinners:
+    """Rank 0's winners array, addressable by every rank's kernels (CUDA IPC).
+
+    `ptr(b0)` is the device address a rank passes to ap_collage_run as
+    winners_dev (with flags AP_COLLAGE_ACCUMULATE | AP_COLLAGE_SYSTEM) for
+    its partition starting at block b0.  Per step: `begin(stream)` on every
+    rank (rank 0 sets the sentinels, all ranks wait for it), the ranks' kernels
+    accumulate, `end()` on every rank; then rank 0's `result` holds the
+    combined winners."""
+
+    def __init__(self, ap, nblocks, rank, world, dist, device):
+        import torch
+        self.ap, self.rank, self.world, self.dist = ap, rank, world, dist
+        self.nblocks = nblocks
+        self.result = None
+        self._mapped = None
+        if rank == 0:
+            self.result = torch.empty((nblocks, 2), dtype=torch.int32, device=device)
+            blob = [bytes(ap.ap_ipc_export(self.result))] if world > 1 else [None]
+        else:
+            blob = [None]
+        if world > 1:
+            dist.broadcast_object_list(blob, src=0)
+        if rank == 0:
+            self._base = self.result.data_ptr()
+        else:
+            h = ap.ap_ipc_handle_t.from_buffer_copy(blob[0])
+            self._mapped = ap.ap_ipc_import(h, device.index if device.index is not None else 0)
+            self._base = self._mapped
+
+    def ptr(self, b0=0):
+        return self._base + 8 * b0
+
+    def begin(self, stream=None):
+        import torch
+        if self.rank == 0:
+            self.ap.ap_winners_init(self.result, self.nblocks, stream)
+            torch.cuda.synchronize()
+        if self.world > 1:
+            self.dist.barrier()
+
+    def end(self):
+        import torch
+        torch.cuda.synchronize()
+        if self.world > 1:
+            self.dist.barrier()
+
+    def close(self):
+        if self._mapped is not None:
+            self.ap.ap_ipc_close(self._mapped)
+            self._mapped = None

@@ -69,8 +69,12 @@ def test_collage_matches_oracle(ap, group, schedule, frames):
         torch.cuda.synchronize()
         assert ap.ap_last_device_error(cache) == 0
         got = win.cpu().numpy().view(np.uint32)
-        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n,
-                              off.cpu().numpy().view(np.uint32), ids.cpu().numpy().view(np.uint32))
+        # the oracle runs on its own index (never on the GPU-built CSR); the
+        # GPU index must equal it bit for bit
+        o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        assert np.array_equal(off.cpu().numpy().view(np.uint32), o_off)
+        assert np.array_equal(ids.cpu().numpy().view(np.uint32), o_ids)
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
         assert np.array_equal(got, want)
         # planted copies found at distance 0
         assert np.all(got[is_copy.astype(bool), 1] == 0)
@@ -291,6 +295,42 @@ def test_collage_record_slices_min_reduce_to_whole(ap, world, chunks):
             with pytest.raises(APError):
                 ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n,
                                                           **bad), part)
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("schedule", [0, 1, 2, 3])
+@pytest.mark.parametrize("group", [1, 8])
+def test_empty_candidate_sets_give_the_sentinel(ap, group, schedule):
+    """R-A4: a block whose L buckets are all empty has no candidate; its
+    winner is (0xFFFFFFFF, 0xFFFFFFFF).  A small dataset spread over 2^14
+    buckets with one table leaves most blocks without candidates (planted
+    copies still find theirs); every schedule must reproduce the oracle,
+    sentinels included, from the oracle's own index."""
+    dev = torch.device("cuda:0")
+    n, stride, w, bb, L, K = 512, 4096, 2500, 14, 1, 8
+    W, H = 256, 256
+    recs, proj, bias, img, src, is_copy = _setup(n, W, H, L, K, w, bb, seed=41)
+    o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+    want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+    empty = np.all(want == oracle.EMPTY, axis=1)
+    assert empty.sum() > 0 and (~empty).sum() > 0, (empty.sum(), len(empty))
+    cache = ap.ap_cache_create(32, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        assert np.array_equal(off.cpu().numpy().view(np.uint32), o_off)
+        assert np.array_equal(ids.cpu().numpy().view(np.uint32), o_ids)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride,
+                                                  group=group, schedule=schedule), win)
+        torch.cuda.synchronize()
+        assert ap.ap_last_device_error(cache) == 0
+        assert np.array_equal(win.cpu().numpy().view(np.uint32), want)
+        assert check_invariants(ap, cache, [r], 32) == []
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)

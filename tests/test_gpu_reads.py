@@ -260,7 +260,9 @@ def test_per_access_deref_kernel(ap, dev, frames):
 def test_seq_tma_staged(ap, dev, prefill, frames, unit):
     """AP_ACCESS_TMA: the SEQ stream staged through shared memory by TMA bulk
     copies, one pin per unit; apointer and raw twin == oracle, resident or
-    faulting (3 frames: every unit evicts, two units pinned per warp at most)."""
+    faulting (3 frames: every unit evicts, two units pinned per warp at most).
+    A launch whose resident warps could pin more than the frames (two units
+    per warp) is refused instead of waiting into the watchdog."""
     page, nbytes = 65536, 16 << 20
     f = make_file(nbytes, seed=41)
     cache = ap.ap_cache_create(frames, page)
@@ -269,7 +271,7 @@ def test_seq_tma_staged(ap, dev, prefill, frames, unit):
         if prefill:
             ap.ap_prefill(cache, r, 0, min(frames, nbytes // page))
             torch.cuda.synchronize()
-        grid, block = (148, 512) if frames > 3 else (1, 32)
+        grid, block = {1024: (148, 512), 24: (1, 256), 3: (1, 32)}[frames]
         cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=unit, passes=2,
                            access=ap.AP_ACCESS_TMA)
         got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
@@ -282,10 +284,71 @@ def test_seq_tma_staged(ap, dev, prefill, frames, unit):
         assert np.array_equal(_run(ap, cache, r, cfg_raw, grid * block, dev).view(np.uint64), want)
         assert check_invariants(ap, cache, [r], frames) == []
         from paper_conf_isca_shaharbs16_b200._lib import APError
+        if frames < min(2 * 148 * 16, nbytes // page):
+            with pytest.raises(APError):  # too few frames for 2 pins per resident warp
+                ap.ap_bench_read(cache, r, ap.bench_cfg(ap.AP_SEQ, 16, 148, 512, unit_bytes=unit,
+                                                        access=ap.AP_ACCESS_TMA),
+                                 torch.zeros(148 * 512, dtype=torch.int64, device=dev))
         with pytest.raises(APError):  # 4-B elements are not staged
             ap.ap_bench_read(cache, r, ap.bench_cfg(ap.AP_SEQ, 4, 1, 32, unit_bytes=unit,
                                                     access=ap.AP_ACCESS_TMA),
                              torch.zeros(32, dtype=torch.int64, device=dev))
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("pattern,elem,page,nbytes,prefill", [
+    (2, 4, 4096, 256 << 20, False),   # C3 shape, cold: every link a major fault
+    (2, 16, 4096, 256 << 20, True),   # resident: every link a minor fault
+    (2, 4, 65536, 512 << 20, False),
+    (1, 4, 65536, 64 << 20, True),    # UNIFORM: lanes of a warp may share pages
+    (1, 16, 4096, 16 << 20, True),
+])
+def test_link_events_closed_form(ap, dev, pattern, elem, page, nbytes, prefill):
+    """O2 closed form: with a cache that
+    never runs out of frames, major + minor faults == the number of (warp,
+    iteration, distinct page) link events computed from the access trace
+    alone (oracle.invariants.link_events) -- one leader per page per warp,
+    DIVERGENT warps (32 distinct pages) and UNIFORM warps (shared pages)."""
+    from oracle import invariants
+    f = make_file(nbytes, seed=31)
+    npages = nbytes // page
+    frames = npages + 8  # never under frame pressure: no downgrade, no eviction
+    cache = ap.ap_cache_create(frames, page)
+    try:
+        r = ap.ap_mmap(cache, f)
+        if prefill:
+            ap.ap_prefill(cache, r, 0, npages)
+            torch.cuda.synchronize()
+        grid, block, reads, seed = 32, 256, 4, 77
+        nthreads = grid * block
+        offs = oracle.offsets(pattern, nbytes, elem, nthreads, reads, seed, page)
+        pg = offs >> np.uint64(page.bit_length() - 1)
+        if not prefill:
+            # cold runs wait on pages other warps are loading, and a waiting
+            # warp may drop links it already holds (R-A19); that can only add
+            # a link when a thread's next read is on the same page, which this
+            # seeded trace never does
+            assert not np.any(pg[:, 1:] == pg[:, :-1])
+        want_links = invariants.link_events(offs, page.bit_length() - 1)
+        st0 = ap.ap_cache_stats(cache)
+        cfg = ap.bench_cfg(pattern, elem, grid, block, reads_per_thread=reads, seed=seed,
+                           page_bytes=page if pattern == 2 else 0)
+        got = _run(ap, cache, r, cfg, nthreads, dev).view(np.uint64)
+        if pattern == 2:
+            want = oracle.read_divergent(f, nbytes, page, elem, nthreads, reads, seed)
+        else:
+            want = oracle.read_uniform(f, nbytes, elem, nthreads, reads, seed)
+        assert np.array_equal(got, want)
+        st1 = ap.ap_cache_stats(cache)
+        assert invariants.check_link_count(st0, st1, want_links) == []
+        if prefill:
+            assert st1["major"] == st0["major"]
+        else:
+            assert st1["major"] - st0["major"] == len(np.unique(pg))  # exactly once per page
+        assert st1["evictions"] == 0
+        assert check_invariants(ap, cache, [r], frames) == []
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)

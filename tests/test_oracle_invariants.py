@@ -1,6 +1,7 @@
 """Pins for O2 (oracle/invariants.py): a consistent dump passes, and a dump
 that breaks each invariant of PAPER.md:113-115/145/157 is rejected."""
 import numpy as np
+import pytest
 
 from oracle import invariants as inv
 
@@ -65,3 +66,65 @@ def test_fill_counts():
     assert inv.check_fill_counts({"major": 11, "evictions": 0}, 10, 16, 16)
     assert inv.check_fill_counts({"major": 9, "evictions": 0}, 10, 4, 16)
     assert inv.check_fill_counts({"major": 30, "evictions": 20}, 10, 4, 16) == []
+
+
+def _link_events_brute(offs, lg):
+    """Listing 1 walked by hand: per warp and iteration,
+    the set of pages whose lanes are not linked to them yet."""
+    n, reads = offs.shape
+    events = 0
+    linked = [None] * n
+    for w in range(n // 32):
+        for i in range(reads):
+            need = set()
+            for lane in range(32):
+                t = 32 * w + lane
+                p = int(offs[t, i]) >> lg
+                if linked[t] != p:
+                    need.add(p)
+                    linked[t] = p
+            events += len(need)
+    return events
+
+
+def test_link_events_closed_forms():
+    """one leader (one link) per distinct page per warp."""
+    from oracle.invariants import link_events
+    lg = 12
+    reads, warps = 5, 3
+    n = 32 * warps
+    # every lane of a warp on the same page, a new page each iteration
+    same = np.array([[((w * 100 + i) << lg) + 4 * (t % 32) for i in range(reads)]
+                     for t in range(n) for w in [t // 32]], dtype=np.uint64)
+    assert link_events(same, lg) == warps * reads
+    # 32 distinct pages per warp-iteration
+    dist = np.array([[((t * 1000 + i) << lg) for i in range(reads)] for t in range(n)],
+                    dtype=np.uint64)
+    assert link_events(dist, lg) == 32 * warps * reads
+    # lanes that stay on their page never link again
+    stay = np.array([[(t << lg) + 8 * i for i in range(reads)] for t in range(n)],
+                    dtype=np.uint64)
+    assert link_events(stay, lg) == 32 * warps
+    # leaving a page and coming back is a new link (the pointer was unlinked)
+    back = np.array([[((i % 2) << lg) for i in range(reads)] for t in range(32)],
+                    dtype=np.uint64)
+    assert link_events(back, lg) == reads
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_link_events_brute_force(seed):
+    from oracle.invariants import link_events
+    rng = np.random.default_rng(seed)
+    offs = rng.integers(0, 1 << 18, size=(64, 7), dtype=np.uint64)  # 64 pages of 4 KiB
+    assert link_events(offs, 12) == _link_events_brute(offs, 12)
+
+
+def test_offsets_match_the_per_read_generator():
+    import oracle
+    for pattern, page in ((1, 0), (2, 4096)):
+        offs = oracle.offsets(pattern, 1 << 22, 4, 64, 3, 5, page)
+        for t in (0, 31, 63):
+            for i in range(3):
+                want = (oracle.uniform_off(1 << 22, 4, 5, t, i) if pattern == 1 else
+                        oracle.divergent_off(1 << 22, page, 4, 5, t, i))
+                assert int(offs[t, i]) == want
