@@ -288,10 +288,10 @@ def run_hit(args, torch, dev, ap, cache, region, f, stream, span=GiB, passes=8):
                          overhead_of_means=float(np.mean(t) / np.mean(tr) - 1))
     t_raw = np.array(t_raw_all)
     res.update(raw_s=float(np.mean(t_raw)), raw_gbs=nbytes / np.mean(t_raw) / 1e9)
-    # per-access form: one load in flight per warp, so it runs at full
-    # occupancy (4 CTAs of 512 per SM); its twin is the same per-access loop
-    # on a raw pointer at the same launch
-    grid_d = 4 * 148
+    # per-access form: `v = *q; q += 32`, AP_DEREF_PIPE dereferences in
+    # flight per lane, one CTA of 512 per SM (the kernel's launch bounds);
+    # its twin is the same per-access loop on a raw pointer at the same launch
+    grid_d = 148
     out_d = torch.empty(grid_d * block, dtype=torch.int64, device=dev)
     out_rd = torch.empty_like(out_d)
     cfg_rd = ap.bench_cfg(ap.AP_SEQ, 16, grid_d, block, unit_bytes=page, passes=passes,
@@ -440,7 +440,8 @@ def emit_c2(args, res_all, rank, world):
                            "headline); range = pin_range (one check per page); deref = `v = *q; "
                            "q += 32` one access at a time (the paper's loop, each access checked "
                            "and able to fault; the loop issues access j+D before it uses access "
-                           "j, D = AP_DEREF_PIPE), overhead_vs_raw is against the tiled raw "
+                           "j, D = AP_DEREF_PIPE = 6, 148 CTAs of 512), overhead_vs_raw is "
+                           "against the tiled raw "
                            "twin, deref_vs_raw_per_access_twin against the identical per-access "
                            "loop on a raw pointer at the same launch",
             "overhead_method": "median over %d alternating (apointer, raw) launch pairs of "
@@ -559,6 +560,10 @@ def main():
                         "default 12 for c4 and c5 (measured: C4 8/12/16 -> 30.3/29.2/29.1 ms, "
                         "C5 8/12/16/24 -> 0.608/0.594/0.598/0.648 s)")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
+    p.add_argument("--combine", default="fused", choices=["fused", "nccl"],
+                   help="collage, N > 1: fold winners into rank 0's array from the kernels "
+                        "(CUDA IPC + system-scope atomics, no collective) or one NCCL "
+                        "gather / MIN reduce after the kernel")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-collage", action="store_true",
                    help="default workload only: skip the embedded C4 collage object")

@@ -49,6 +49,38 @@ def _collage_config(name):
                          "page cache per GPU (cold per step), one NCCL gather of the winners")
 
 
+def numa_interleave(arr):
+    """Spread the pages of a host buffer round-robin over the host's NUMA
+    nodes (mbind MPOL_INTERLEAVE before the first touch), so G GPUs reading
+    the one pinned file over their own PCIe links do not all pull from the
+    memory of one socket (SURVEY.md §7 "Host side at scale").  Returns the
+    node count used (1 = nothing to do or not supported)."""
+    import ctypes
+    try:
+        with open("/sys/devices/system/node/online") as f:
+            spec = f.read().strip()
+        nodes = []
+        for part in spec.split(","):
+            a, _, b = part.partition("-")
+            nodes.extend(range(int(a), int(b or a) + 1))
+    except OSError:
+        return 1
+    if len(nodes) < 2:
+        return 1
+    mask = 0
+    for n in nodes:
+        mask |= 1 << n
+    libc = ctypes.CDLL(None, use_errno=True)
+    page = 4096
+    addr = arr.ctypes.data & ~(page - 1)
+    length = arr.ctypes.data + arr.nbytes - addr
+    nm = ctypes.c_ulong(mask)
+    SYS_mbind, MPOL_INTERLEAVE = 237, 3  # x86_64
+    rc = libc.syscall(SYS_mbind, ctypes.c_void_p(addr), ctypes.c_ulong(length), MPOL_INTERLEAVE,
+                      ctypes.byref(nm), ctypes.c_ulong(max(nodes) + 2), 0)
+    return len(nodes) if rc == 0 else 1
+
+
 def _shm_records(cfg, rank, world, dist):
     """The record file in /dev/shm, generated once (all ranks map the same
     pages; each rank registers them for its own GPU)."""
@@ -62,6 +94,7 @@ def _shm_records(cfg, rank, world, dist):
         with open(path, "r+b") as fh:
             mm = mmap.mmap(fh.fileno(), nbytes)
             arr = np.frombuffer(mm, dtype=np.uint8)
+            numa_interleave(arr)  # before the first touch
             chunk = 1 << 18
             for first in range(0, cfg["N"], chunk):
                 cnt = min(chunk, cfg["N"] - first)
@@ -140,12 +173,30 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
                         schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0,
                         id_chunks=id_chunks, id_begin=i0, id_end=i1)
 
+    # N > 1, fused (default): every rank's kernel folds its winners into rank
+    # 0's array over NVLink (CUDA IPC + system-scope atomic min), no
+    # collective; --combine nccl: one NCCL gather / MIN reduce after the kernel
+    fused = world > 1 and getattr(args, "combine", "fused") == "fused"
+    sw = mgpu.SharedWinners(ap, nb, rank, world, dist, dev) if fused else None
+    inp_f = None
+    if fused:
+        inp_f = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
+                              cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
+                              block_count=b1 - b0, schedule=args.schedule, unit_begin=u0,
+                              unit_count=u1 - u0, id_chunks=id_chunks, id_begin=i0, id_end=i1,
+                              flags=ap.AP_COLLAGE_ACCUMULATE | ap.AP_COLLAGE_SYSTEM)
+
     def combine():
+        if fused:
+            return sw.result
         if bucket:
             return mgpu.reduce_winners_min(win, rank, world, dist)  # one NCCL reduce (S12)
         return mgpu.gather_winners(win, rank, world, dist, nb)  # one NCCL gather (S12)
 
     def step():
+        if fused:
+            ap.ap_collage_run(cache, region, inp_f, sw.ptr(b0), stream)
+            return
         ap.ap_collage_run(cache, region, inp, win, stream)
         if world > 1:
             combine()
@@ -153,18 +204,31 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     link = host_link_peak(torch, dev)
     for _ in range(args.warmup):
         ap.ap_cache_reset(cache)
-        if world > 1:
+        if fused:
+            sw.begin(stream)
+        elif world > 1:
             dist.barrier()
         timed(torch, step, stream)
+        if fused:
+            sw.end()
     times, stats = [], []
     with ClockSampler(torch.cuda.current_device()) as clk:
         for _ in range(args.steps):
             ap.ap_cache_reset(cache)  # cold cache each step (untimed)
-            if world > 1:
+            if fused:
+                sw.begin(stream)  # rank 0 sets the sentinels; all ranks start together
+            elif world > 1:
                 dist.barrier()
             torch.cuda.synchronize()
             times.append(timed(torch, step, stream))
+            if fused:
+                sw.end()  # every rank's folds are in rank 0's array
             stats.append(ap.ap_cache_stats(cache))
+    if fused:
+        # this rank's own share, for the comparisons below
+        ap.ap_cache_reset(cache)
+        ap.ap_collage_run(cache, region, inp, win, stream)
+        torch.cuda.synchronize()
     err = ap.ap_last_device_error(cache)
     got = win.cpu().numpy().view(np.uint32).copy()
     # the other schedules, for comparison (cold cache, same winners)
@@ -261,6 +325,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         e2e.append(s.elapsed_time(e) * 1e-3)
     cands = None
     res = dict(cfg=cfg, id_chunks=id_chunks, times=times, stats=stats, err=err, got=got, b0=b0, b1=b1, nb=nb,
+               fused=fused,
                units=(u0, u1), bucket=bucket, records=bool(i1),
                other=other_res,
                link=link, raw=raw, e2e=e2e, clocks=clk.summary(), t_gen=t_gen, t_pin=t_pin,
@@ -270,6 +335,8 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     res["parity"] = None
     # the combined answer (N > 1) on rank 0
     full = combine() if world > 1 else None
+    if sw is not None:
+        sw.close()
     if bucket and rank == 0:
         got = full.cpu().numpy().view(np.uint32).copy()  # rank 0's own array is partial
         res["got"] = got
@@ -343,11 +410,17 @@ def emit_collage(args, res_all, world, METRIC):
                    "schedule": SCHED_NAMES[args.schedule],
                    "id_chunks": r0["id_chunks"],
                    "l2": "inputs larger than L2 (multi-GB record file, cold cache per step)",
-                   "parallelism": ((f"record-id slices (file shards) over {world} ranks, all units "
-                                    "each + NCCL MIN reduce") if r0.get("records") else
-                                   f"(table, bucket) units partitioned over {world} ranks + NCCL "
-                                   "MIN reduce" if r0.get("bucket") else
-                                   f"blocks partitioned over {world} rank(s) + NCCL gather")},
+                   "parallelism": (((f"record-id slices (file shards) over {world} ranks, all units "
+                                     "each") if r0.get("records") else
+                                    f"(table, bucket) units partitioned over {world} ranks"
+                                    if r0.get("bucket") else
+                                    f"blocks partitioned over {world} rank(s)") +
+                                   ("" if world == 1 else
+                                    " + winners folded into rank 0's array by the kernels "
+                                    "(CUDA IPC, system-scope atomic min; no collective)"
+                                    if r0.get("fused") else
+                                    " + NCCL MIN reduce" if r0.get("bucket") else
+                                    " + NCCL gather"))},
         "collage": {"blocks_rank0": r0["b1"] - r0["b0"],
                     "units_rank0": (r0["units"][1] - r0["units"][0]) if r0.get("bucket") else None,
                     "major_faults": st["major"],

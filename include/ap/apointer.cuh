@@ -72,10 +72,14 @@
 #endif
 #endif
 
-/* Speculative load of the hit path; -DAP_SPECULATIVE=0 is
- * the ablation that loads only after the warp's vote. */
+/* Speculative load of the hit path: 1 = the load issues
+ * with the vote (unready lanes read the region descriptor); 0 (default on
+ * B200) = it issues after the vote.  Measured on B200: the per-access loop
+ * keeps several dereferences in flight, so the address select costs more
+ * than the latency it hides (deref overhead vs the raw twin +40 % -> +20 %,
+ * DESIGN.md §5). */
 #ifndef AP_SPECULATIVE
-#define AP_SPECULATIVE 1
+#define AP_SPECULATIVE 0
 #endif
 /* Reference bit of a freshly filled page (second-chance clock, R-A11):
  * 1 = set at the fill, 0 = set only when the page is linked again (a minor
@@ -1127,39 +1131,55 @@ __device__ AP_SLOW_ATTR slow_out<T> store_slow(unsigned m, uint64_t x, uint64_t 
 /* ======================================================================
  * ap::ptr<T> — the apointer (M1; Fig. 3).
  * States: uninitialised (r == nullptr), unlinked (valid bit
- * clear: x is the file offset), linked (valid bit set: x is the address of
- * the datum in its frame, which is pinned by the page's reference count). */
+ * clear: x is the file offset), linked (valid bit set: the lane holds a
+ * reference on file page `page`, whose frame starts at fb; x is the device
+ * address of the datum, fb + its offset from the frame start).
+ *
+ * Where the translation is checked (B200 design): arithmetic
+ * only moves x -- `p += d` is one 64-bit add, no vote, no branch -- and the
+ * dereference checks that x still lies in the linked frame (its page bits
+ * equal fb's).  A pointer that walked off its page still holds that page
+ * until its next dereference (or release / assignment / destruction), where
+ * the fault path unlinks it, warp-aggregated, before linking the new page:
+ * the same Fig. 4 transitions with the unlink deferred to the
+ * next use.  The hit path is then: a 32-bit frame compare, one vote, a load;
+ * and arithmetic costs what it costs on a raw pointer. */
 template <class T>
 struct ptr {
     static_assert(sizeof(T) == 4 || sizeof(T) == 8 || sizeof(T) == 16, "T must be 4/8/16 B");
-    uint64_t x;          /* translation field (R-A16)                       */
-    const dev_region* r; /* metadata: region                                */
-    uint64_t page;       /* metadata: linked page                           */
-    uint32_t lg;         /* metadata: log2(page size)                       */
-    int64_t step = 0;    /* bytes of the last += (stride predictor)         */
+    uint64_t x;          /* translation field (R-A16)                            */
+    uint64_t fb;         /* linked: XL_VALID [| XL_DIRTY] | frame base address;  *
+                          * else XL_VALID (never in x's frame)                   */
+    const dev_region* r; /* metadata: region                                     */
+    uint64_t page;       /* metadata: the page a linked lane holds               */
+    uint32_t lg;         /* metadata: log2(page size)                            */
+    int64_t step = 0;    /* bytes of the last += (stride predictor)              */
 
-    __device__ __forceinline__ ptr() : x(0), r(nullptr), page(0), lg(12) {}
+    __device__ __forceinline__ ptr() : x(0), fb(XL_VALID), r(nullptr), page(0), lg(12) {}
     __device__ __forceinline__ ptr(const dev_region* reg, uint32_t log2_page, uint64_t foff)
-        : x(foff), r(reg), page(0), lg(log2_page) {}
+        : x(foff), fb(XL_VALID), r(reg), page(0), lg(log2_page) {}
     /* Copy: the copy starts unlinked (Fig. 4). */
-    __device__ __forceinline__ ptr(const ptr& o) : x(o.foff()), r(o.r), page(0), lg(o.lg) {}
+    __device__ __forceinline__ ptr(const ptr& o)
+        : x(o.foff()), fb(XL_VALID), r(o.r), page(0), lg(o.lg) {}
     __device__ __forceinline__ ptr& operator=(const ptr& o) {
         const uint64_t nx = o.foff();
         release();
         x = nx;
+        fb = XL_VALID;
         r = o.r;
         lg = o.lg;
         return *this;
     }
     /* Move: the same pointer changes hands -- its link moves with it, no
      * reference count changes. */
-    __device__ __forceinline__ ptr(ptr&& o) : x(o.x), r(o.r), page(o.page), lg(o.lg) {
+    __device__ __forceinline__ ptr(ptr&& o) : x(o.x), fb(o.fb), r(o.r), page(o.page), lg(o.lg) {
         o.detach();
     }
     __device__ __forceinline__ ptr& operator=(ptr&& o) {
         if (this == &o) return *this;
         release();
         x = o.x;
+        fb = o.fb;
         r = o.r;
         page = o.page;
         lg = o.lg;
@@ -1168,54 +1188,88 @@ struct ptr {
     }
     __device__ __forceinline__ ~ptr() { release(); }
 
-    /* the valid bit is the sign of the translation's high word: one compare */
-    __device__ __forceinline__ bool linked() const { return (int32_t)(uint32_t)(x >> 32) < 0; }
+    /* the lane holds a reference on `page` (valid bit: the sign of x's high word) */
+    __device__ __forceinline__ bool holds() const { return (int32_t)(uint32_t)(x >> 32) < 0; }
+    /* linked and still inside the linked frame: the hit path's check */
+    __device__ __forceinline__ bool in_frame(uint64_t a) const {
+        return (uint32_t)(a >> 32) == (uint32_t)(fb >> 32) &&
+               (((uint32_t)a ^ (uint32_t)fb) >> lg) == 0;
+    }
+    __device__ __forceinline__ bool ready() const { return in_frame(x); }
+    /* kept for callers of the previous API: linked = ready to dereference */
+    __device__ __forceinline__ bool linked() const { return ready(); }
     /* File offset (xAddress) the pointer designates, linked or not. */
     __device__ __forceinline__ uint64_t foff() const {
-        return linked() ? ((page << lg) | (x & ((1ull << lg) - 1))) : x;
+        return holds() ? (page << lg) + (uint64_t)((int64_t)(x & XL_ADDR) - (int64_t)(fb & XL_ADDR))
+                       : x;
     }
 
     /* S3: dereference (hit path inline, fault path out of line). */
     __device__ __forceinline__ T operator*() {
         const unsigned m = __activemask();
-        const bool v = linked();
 #if AP_SPECULATIVE
+        /* speculative load: lanes off their frame load the
+         * region descriptor (always mapped) while the warp votes */
+        const bool v = ready();
         const T* a = v ? reinterpret_cast<const T*>(x & XL_ADDR) : reinterpret_cast<const T*>(r);
-        T val = detail::ld_data<T>(a); /* speculative prefetch */
+        T val = detail::ld_data<T>(a);
+        if (__all_sync(m, v)) return val;
 #else
-        /* ablation: the load waits for the vote */
-        if (__all_sync(m, v)) return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
-        T val{};
+        /* the load issues after the vote: on B200 the per-access loop keeps
+         * several dereferences in flight, so the select the speculative
+         * address needs costs more than the latency it hides */
+        if (__all_sync(m, ready())) return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
 #endif
 #if AP_PREFETCH_DIST > 0
         {
-            /* stride prefetch: the datum AP_PREFETCH_DIST steps ahead, if it
-             * is in the linked page, is requested into L2 (no register
-             * result, so nothing waits on it) */
             const uint64_t px = x + (uint64_t)(step * AP_PREFETCH_DIST);
-            if (v && ((x ^ px) >> lg) == 0) detail::prefetch_l2(reinterpret_cast<const void*>(px & XL_ADDR));
+            if (in_frame(px)) detail::prefetch_l2(reinterpret_cast<const void*>(px & XL_ADDR));
         }
 #endif
-        if (__all_sync(m, v)) return val;
-        if (detail::try_link_minor<T>(m, x, page, r, lg))
+        return deref_miss(m);
+    }
+
+    /* The pointer's miss path: lanes that walked off their frame unlink it
+     * (warp-aggregated), then unlinked lanes link -- inline when the page is
+     * resident (link_minor), else through the fault handler. */
+    __device__ __forceinline__ T deref_miss(unsigned m) {
+        drop_stale(m);
+        if (detail::try_link_minor<T>(m, x, page, r, lg)) {
+            sync_fb();
             return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
+        }
         const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
         x = o.x;
         page = o.page;
+        sync_fb();
         return o.val;
+    }
+
+    /* The same, but a thread that holds a second pointer `other` releases it
+     * first when this dereference must fault on a recycled cache (R-A19:
+     * never wait for a frame while pinning one); the check costs nothing on
+     * the hit path. */
+    template <class U>
+    __device__ __forceinline__ T deref_releasing(ptr<U>& other) {
+        const unsigned m = __activemask();
+        if (__all_sync(m, ready())) return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
+        if (cache_pressure()) other.release();
+        return deref_miss(m);
     }
 
     /* Store through the pointer (writable mappings; Fig. 3 `*ptr = 25`). */
     __device__ __forceinline__ void store(const T& v) {
         const unsigned m = __activemask();
-        const bool ok = (x & (XL_VALID | XL_DIRTY)) == (XL_VALID | XL_DIRTY);
+        const bool ok = ready() && (x & XL_DIRTY);
         if (__all_sync(m, ok)) {
             detail::st_data<T>(reinterpret_cast<T*>(x & XL_ADDR), v);
             return;
         }
+        drop_stale(m);
         const detail::slow_out<T> o = detail::store_slow<T>(m, x, page, r, v);
         x = o.x;
         page = o.page;
+        sync_fb();
     }
 
     /* Tiled store: p[k * stride] = v[k] for k < N, p unchanged.  One check
@@ -1225,8 +1279,7 @@ struct ptr {
     __device__ __forceinline__ void write_tile(const T (&v)[N], int64_t stride) {
         const unsigned m = __activemask();
         const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
-        const bool ok = (x & (XL_VALID | XL_DIRTY)) == (XL_VALID | XL_DIRTY) &&
-                        ((x ^ (x + span)) >> lg) == 0;
+        const bool ok = ready() && (x & XL_DIRTY) && in_frame(x + span);
         if (__all_sync(m, ok)) {
             T* a = reinterpret_cast<T*>(x & XL_ADDR);
 #pragma unroll
@@ -1251,19 +1304,19 @@ struct ptr {
         p -= N * stride;
     }
 
-    /* warp-wide: every active lane is linked (and, for stores, marked dirty) */
-    __device__ __forceinline__ bool linked_all() const { return __all_sync(__activemask(), linked()); }
+    /* warp-wide: every active lane is ready (and, for stores, marked dirty) */
+    __device__ __forceinline__ bool linked_all() const { return __all_sync(__activemask(), ready()); }
     __device__ __forceinline__ bool store_ready() const {
-        return __all_sync(__activemask(), (x & (XL_VALID | XL_DIRTY)) == (XL_VALID | XL_DIRTY));
+        return __all_sync(__activemask(), ready() && (x & XL_DIRTY));
     }
 
-    /* p[i] without moving p: a linked lane whose target stays in the page
+    /* p[i] without moving p: a lane whose target stays in its linked frame
      * reads directly; otherwise a temporary pointer takes the fault. */
     __device__ __forceinline__ T operator[](int64_t i) {
         const unsigned m = __activemask();
         const uint64_t nb = (uint64_t)(i * (int64_t)sizeof(T));
         const uint64_t nx = x + nb;
-        const bool in = linked() && ((x ^ nx) >> lg) == 0;
+        const bool in = in_frame(nx);
         const T* a = in ? reinterpret_cast<const T*>(nx & XL_ADDR) : reinterpret_cast<const T*>(r);
         T val = detail::ld_data<T>(a);
         if (__all_sync(m, in)) return val;
@@ -1274,31 +1327,27 @@ struct ptr {
 
     /* Tiled read: v[k] = p[k * stride] for k < N, p unchanged.  One
      * translation check covers the whole tile when every lane is linked and
-     * its tile stays inside its page; the N loads then issue back to back
+     * its tile stays inside its frame; the N loads then issue back to back
      * (memory tiling; one check per tile instead of per access
      * is the hand-written form of the check elimination PAPER.md:450 asks of
-     * a compiler).  An unlinked pointer is first linked by dereferencing its
-     * first element (the usual fault path); a tile that straddles a page is
-     * read element by element.  No loaded value is ever live across a call
-     * into the fault path, so the tile stays in registers. */
+     * a compiler).  Otherwise the pointer is (re)linked through the fault
+     * path; a tile that straddles a page is read element by element.  No
+     * loaded value is ever live across a call into the fault path. */
     template <int N>
     __device__ __forceinline__ void read_tile(T (&v)[N], int64_t stride) {
         const unsigned m = __activemask();
         const uint64_t span = (uint64_t)((N - 1) * stride * (int64_t)sizeof(T));
-        bool ok = linked() && ((x ^ (x + span)) >> lg) == 0;
+        bool ok = ready() && in_frame(x + span);
         if (__builtin_expect(!__all_sync(m, ok), 0)) {
-            if (__any_sync(m, !linked()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
-                const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
-                x = o.x;
-                page = o.page;
-            }
-            ok = linked() && ((x ^ (x + span)) >> lg) == 0;
+            relink(m);
+            ok = ready() && in_frame(x + span);
             if (!__all_sync(m, ok)) {
                 /* some lane's tile straddles a page */
                 const detail::tile_out<T, N> t = detail::read_tile_slow<T, N>(m, x, page, r, lg, stride);
 #pragma unroll
                 for (int k = 0; k < N; ++k) v[k] = t.v[k];
                 x = t.x;
+                fb = XL_VALID;
                 return;
             }
         }
@@ -1310,22 +1359,19 @@ struct ptr {
     /* Translate once for a whole range: make the pointer linked and return
      * its direct device address if [p, p + bytes) of every lane lies inside
      * the page that lane links (else nullptr, nothing changed but a link).
-     * The address stays valid while this pointer stays linked -- a linked
+     * The address stays valid while this pointer keeps its link -- a linked
      * pointer keeps its page active and its mapping fixed (PAPER.md:113,
-     * 141) -- so a loop can stream through it with plain loads.  This is the
-     * per-page hoisting of the translation check that PAPER.md:450 expects
-     * from compiler support. */
+     * 141) -- i.e. until it is released, assigned, destroyed or dereferenced
+     * after moving off the page; a loop can stream through it with plain
+     * loads.  This is the per-page hoisting of the translation check that
+     * PAPER.md:450 expects from compiler support. */
     __device__ __forceinline__ const T* pin_range(uint64_t bytes) {
         const unsigned m = __activemask();
         const uint64_t last = bytes ? bytes - 1 : 0;
-        bool ok = linked() && ((x ^ (x + last)) >> lg) == 0;
+        bool ok = ready() && in_frame(x + last);
         if (!__all_sync(m, ok)) {
-            if (__any_sync(m, !linked()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
-                const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
-                x = o.x;
-                page = o.page;
-            }
-            ok = linked() && ((x ^ (x + last)) >> lg) == 0;
+            relink(m);
+            ok = ready() && in_frame(x + last);
             if (!__all_sync(m, ok)) return nullptr;
         }
         return reinterpret_cast<const T*>(x & XL_ADDR);
@@ -1333,15 +1379,16 @@ struct ptr {
 
     /* Split-phase link -- a translation prefetch, the overlap of PAPER.md:195
      * ("access memory in parallel with checking") applied to the minor fault:
-     * link_begin() groups the unlinked lanes by page (S5) and issues each
-     * group's optimistic PTE add (S6, relaxed: the frame data is then read
-     * with .cg loads whose addresses depend on the add's result) without
+     * link_begin() groups the lanes that hold no page by page (S5) and issues
+     * each group's optimistic PTE add (S6, relaxed: the frame data is then
+     * read with .cg loads whose addresses depend on the add's result) without
      * waiting for it; link_finish(t) consumes it and links the lanes whose
      * page was resident (a non-resident page's add is undone; those lanes
      * stay unlinked and take the ordinary fault path on their next
-     * dereference).  Contract: between the two calls the warp must not enter
-     * the fault path; loads through pointers already linked, arithmetic and
-     * unlinks are fine.  Every link_begin is followed by its link_finish. */
+     * dereference).  Lanes that still hold a page are left alone.  Contract:
+     * between the two calls the warp must not enter the fault path; loads
+     * through pointers already linked, arithmetic and unlinks are fine.
+     * Every link_begin is followed by its link_finish. */
     struct link_ticket {
         uint64_t old; /* leader: the PTE before the add */
         unsigned grp; /* this lane's page group         */
@@ -1349,7 +1396,7 @@ struct ptr {
     };
     __device__ __forceinline__ link_ticket link_begin() {
         const unsigned m = __activemask();
-        const bool need = !linked() && x + sizeof(T) <= r->bytes && (x % sizeof(T)) == 0;
+        const bool need = !holds() && x + sizeof(T) <= r->bytes && (x % sizeof(T)) == 0;
         const uint64_t pg = x >> lg;
         const unsigned grp =
             __match_any_sync(m, need ? (((unsigned long long)r->id << 48) | pg) : ~0ull);
@@ -1393,31 +1440,19 @@ struct ptr {
             const uint64_t f = (old >> 32) & PTE_FRAME_MASK;
             x = XL_VALID | ((uint64_t)(r->pool + f * P) + (x & (P - 1)));
             page = pg;
+            sync_fb();
         }
     }
 
-    /* S4: arithmetic.  Staying inside the page keeps the link; leaving it
-     * unlinks with a warp-aggregated decrement (S10). */
+    /* S4: arithmetic moves the pointer and nothing else (one 64-bit add):
+     * leaving the page is noticed, and the page unlinked (S10), by the next
+     * dereference.  A step of a terabyte or more unlinks at once, so an
+     * address never wraps into the flag bits. */
     __device__ __forceinline__ ptr& operator+=(int64_t d) {
         const uint64_t nb = (uint64_t)(d * (int64_t)sizeof(T));
         step = (int64_t)nb;
-        const uint64_t nx = x + nb;
-        /* A step shorter than the smallest page (4 KiB) leaves the page iff
-         * the page bits of the low word change (a carry into the high word
-         * flips bits lg..31 too, lg <= 21): a 32-bit test.  With a constant
-         * stride the compiler keeps only that branch. */
-        bool cross;
-        if (nb + 4095u < 8191u)
-            cross = linked() && (((uint32_t)x ^ (uint32_t)nx) >> lg) != 0;
-        else
-            cross = linked() && ((x ^ nx) >> lg) != 0;
-        const unsigned m = __activemask();
-        if (__any_sync(m, cross)) {
-            detail::unlink_lanes(m, cross, r, page);
-            x = cross ? ((page << lg) | (x & ((1ull << lg) - 1))) + nb : nx;
-        } else {
-            x = nx;
-        }
+        if (nb + (1ull << 40) >= (1ull << 41)) release();
+        x += nb;
         return *this;
     }
     __device__ __forceinline__ ptr& operator-=(int64_t d) { return *this += -d; }
@@ -1441,16 +1476,50 @@ struct ptr {
     /* Unlink now (also done by the destructor and by assignment). */
     __device__ __forceinline__ void release() {
         const unsigned m = __activemask();
-        const bool l = linked();
+        const bool l = holds();
         if (__any_sync(m, l)) {
+            const uint64_t off = foff();
             detail::unlink_lanes(m, l, r, page);
-            if (l) x = (page << lg) | (x & ((1ull << lg) - 1));
+            if (l) {
+                x = off;
+                fb = XL_VALID;
+            }
         }
     }
 
    private:
+    /* frame base of a linked lane (its dirty bit included), else XL_VALID */
+    __device__ __forceinline__ void sync_fb() {
+        fb = holds() ? (x & ~((1ull << lg) - 1)) : XL_VALID;
+    }
+    /* lanes that walked off their frame unlink it and carry
+     * on unlinked at the same file offset */
+    __device__ __forceinline__ void drop_stale(unsigned m) {
+        const bool stale = holds() && !ready();
+        if (__any_sync(m, stale)) {
+            const uint64_t off = foff();
+            detail::unlink_lanes(m, stale, r, page);
+            if (stale) {
+                x = off;
+                fb = XL_VALID;
+            }
+        }
+    }
+    /* make every lane of m linked at its current offset */
+    __device__ __forceinline__ void relink(unsigned m) {
+        drop_stale(m);
+        if (__any_sync(m, !holds()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
+            const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
+            x = o.x;
+            page = o.page;
+        }
+        sync_fb();
+    }
     /* Forget the link without touching the count (it moved elsewhere). */
-    __device__ __forceinline__ void detach() { x = foff(); }
+    __device__ __forceinline__ void detach() {
+        x = foff();
+        fb = XL_VALID;
+    }
 };
 
 /* gvmmap (M17): an unlinked apointer to byte offset

@@ -124,13 +124,14 @@ __device__ __forceinline__ unsigned long long work_elem(const uint4& v, const ui
  * access j + D is dereferenced (and its pointer moved on) before the value of
  * access j is used, so no check or fault of a later access waits for an
  * earlier access's data (the same source for both pointer types).  Built
- * for AP_COMPUTE_MINB CTAs of 512 threads per SM (2 = 64 registers, the
- * paper's budget). */
+ * for AP_COMPUTE_MINB CTAs of 512 threads per SM (1 = 128 registers: at the
+ * Fig. 6 sweep's 148 thread blocks, 16 warps per SM, each with 8 reads in
+ * flight). */
 #ifndef AP_COMPUTE_MINB
-#define AP_COMPUTE_MINB 2
+#define AP_COMPUTE_MINB 1
 #endif
 #ifndef AP_COMPUTE_PIPE
-#define AP_COMPUTE_PIPE 4
+#define AP_COMPUTE_PIPE 8
 #endif
 /* ADD keeps two values per access in the ring */
 #ifndef AP_COMPUTE_PIPE_ADD
@@ -143,15 +144,16 @@ template <class T, int WORK>
 struct ap_access {
     ap::ptr<T> q, q2;
     __device__ __forceinline__ void next(T& v, T& v2) {
-        /* ADD holds two pointers: never fault one while the other pins a
-         * frame of a recycled cache (R-A19) */
-        if (WORK == 0 && !q.linked_all() && q.cache_pressure()) q2.release();
-        v = *q;
-        q += 32;
         if (WORK == 0) {
-            if (!q2.linked_all() && q2.cache_pressure()) q.release();
-            v2 = *q2;
+            /* ADD holds two pointers: never fault one while the other pins a
+             * frame of a recycled cache (R-A19); checked on the miss path */
+            v = q.deref_releasing(q2);
+            q += 32;
+            v2 = q2.deref_releasing(q);
             q2 += 32;
+        } else {
+            v = *q;
+            q += 32;
         }
     }
 };

@@ -87,4 +87,14 @@ void ap_note_cuda_error(cudaError_t e, const char* what, const char* file, int l
 void* ap_scratch(ap_cache_s* c, size_t bytes);
 bool ap_region_ok(const ap_cache_s* c, ap_region_t r);
 
+/* ap_sort.cu: stable LSD radix sort of n (key, value) pairs by the low
+ * `bits` bits of the key (8-bit digits).  The passes ping-pong between
+ * (keys, vals) and (keys_alt, vals_alt); *in_alt tells where the result
+ * is.  scratch: ap_sort_scratch_bytes(n) bytes of device memory.
+ * Asynchronous on s. */
+size_t ap_sort_scratch_bytes(uint64_t n);
+template <class K>
+int ap_sort_pairs(K* keys, K* keys_alt, uint32_t* vals, uint32_t* vals_alt, uint64_t n, int bits,
+                  void* scratch, cudaStream_t s, bool* in_alt);
+
 #endif

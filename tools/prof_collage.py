@@ -19,7 +19,8 @@ N = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 20
 groups = [int(g) for g in sys.argv[2:]] or [4]
 steps = int(os.environ.get("AP_PROF_STEPS", 5))
 W = H = 1024
-L, K, bb, w, page, stride = 4, 8, 14, 60000, 4096, 4096
+stride_env = int(os.environ.get("AP_PROF_STRIDE", 4096))
+L, K, bb, w, page, stride = 4, 8, 14, 60000, 4096, stride_env
 dev = torch.device("cuda:0")
 stream = torch.cuda.current_stream()
 
@@ -63,7 +64,7 @@ def timed(fn):
     return min(ts)
 
 
-for sched in (1, 0):
+for sched in [int(x) for x in os.environ.get("AP_PROF_SCHEDS", "1,0").split(",")]:
     for g in groups:
         mk = lambda mode, rb: ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, N, stride, group=g,  # noqa: E731
                                             block_begin=0, block_count=nb, mode=mode, raw_base=rb,
