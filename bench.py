@@ -560,6 +560,9 @@ def main():
                         "default 12 for c4 and c5 (measured: C4 8/12/16 -> 30.3/29.2/29.1 ms, "
                         "C5 8/12/16/24 -> 0.608/0.594/0.598/0.648 s)")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
+    p.add_argument("--policy", default=None, choices=["clock", "sequential"],
+                   help="c1/c3 eviction policy (default: sequential drop-behind for the "
+                        "single-pass c1 stream, clock otherwise)")
     p.add_argument("--combine", default="fused", choices=["fused", "nccl"],
                    help="collage, N > 1: fold winners into rank 0's array from the kernels "
                         "(CUDA IPC + system-scope atomics, no collective) or one NCCL "

@@ -55,6 +55,12 @@ def run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler, host_lin
                            reads_per_thread=cfg["reads"], page_bytes=cfg["page"], seed=77,
                            mode=ap.AP_MODE_RAW, raw_base=ap.ap_region_devptr(cache, region))
         reads = nthreads * cfg["reads"]
+    # eviction policy: C1 is a single-pass stream, so the drop-behind hint
+    # (AP_POLICY_SEQUENTIAL) by default; the clock alone is measured beside it
+    pol_names = {"clock": ap.AP_POLICY_CLOCK, "sequential": ap.AP_POLICY_SEQUENTIAL}
+    policy = args.policy or ("sequential" if cfg["name"] == "c1" else "clock")
+    ap.ap_cache_set_policy(cache, pol_names[policy])
+    cfg["policy"] = policy
     link = host_link_peak(torch, dev)
     step = lambda: ap.ap_bench_read(cache, region, bc, out, stream)  # noqa: E731
     for _ in range(args.warmup):
@@ -71,6 +77,21 @@ def run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler, host_lin
             stats.append(ap.ap_cache_stats(cache))
     err = ap.ap_last_device_error(cache)
     got = out.cpu().numpy()
+    other = {}
+    for name, pol in pol_names.items():
+        if name == policy:
+            continue
+        ap.ap_cache_set_policy(cache, pol)
+        out_o = torch.empty_like(out)
+        to = []
+        for _ in range(3):
+            ap.ap_cache_reset(cache)
+            to.append(timed(torch, lambda: ap.ap_bench_read(cache, region, bc, out_o, stream),
+                            stream))
+        so = ap.ap_cache_stats(cache)
+        other[name] = dict(s=min(to), fill_GBps=so["fill_bytes"] / min(to) / 1e9,
+                           evictions=so["evictions"], equal=bool(torch.equal(out_o, out)))
+        ap.ap_cache_set_policy(cache, pol_names[policy])
     out_raw = torch.empty_like(out)
     raw_t = min(timed(torch, lambda: ap.ap_bench_read(cache, region, raw, out_raw, stream), stream)
                 for _ in range(3))
@@ -93,7 +114,8 @@ def run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler, host_lin
     ap.ap_munmap(cache, region)
     ap.ap_cache_destroy(cache)
     return dict(cfg=cfg, times=times, stats=stats, err=err, link=link, raw_t=raw_t,
-                raw_equal=raw_equal, reads=reads, clocks=clk.summary(), parity=parity)
+                raw_equal=raw_equal, reads=reads, clocks=clk.summary(), parity=parity,
+                other_policies=other)
 
 
 def emit_reads(args, res_all, world, METRIC):
@@ -112,6 +134,7 @@ def emit_reads(args, res_all, world, METRIC):
         "config": {"workload": cfg["workload"], "file_bytes": cfg["file_bytes"],
                    "page_bytes": cfg["page"], "frames": cfg["frames"], "grid": cfg["grid"],
                    "block": cfg["block"], "reads_per_step": r0["reads"],
+                   "eviction_policy": cfg["policy"],
                    "l2": "cold cache per step; file > L2" if cfg["name"] == "c3" else
                          "cold cache per step (16 MiB file fits L2: C1 measures the fault path)",
                    "parallelism": f"replicas x{world}"},
@@ -123,7 +146,10 @@ def emit_reads(args, res_all, world, METRIC):
                         "evictions": st["evictions"], "waits": st["waits"],
                         "downgrades": st["downgrades"], "nofree": st["nofree"],
                         "raw_zero_copy_twin_s": round(r0["raw_t"], 6),
-                        "raw_twin_equal": r0["raw_equal"], "device_error": r0["err"]},
+                        "raw_twin_equal": r0["raw_equal"], "device_error": r0["err"],
+                        "other_policies": {k: {kk: (round(vv, 6) if isinstance(vv, float) else vv)
+                                               for kk, vv in v.items()}
+                                           for k, v in r0.get("other_policies", {}).items()}},
         "roofline": {"bound": "host_link", "achieved": round(st["fill_bytes"] / t0 / 1e9, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
                      "frac": round(st["fill_bytes"] / t0 / 1e9 / r0["link"], 4), "traffic": None,

@@ -171,6 +171,12 @@ int ap_cache_reset(ap_cache_t cache);
  *                     depend on eviction order)                         */
 #define AP_POLICY_CLOCK 0
 #define AP_POLICY_RANDOM 1
+/*   AP_POLICY_SEQUENTIAL  the clock, plus drop-behind: a warp that faults
+ *                     right after its pointer left a page first reuses that
+ *                     page's frame when no other pointer holds it (a hint for
+ *                     single-pass streams, like MADV_SEQUENTIAL; pages that
+ *                     are read again are better served by the plain clock) */
+#define AP_POLICY_SEQUENTIAL 2
 int ap_cache_set_policy(ap_cache_t cache, int policy, uint64_t seed);
 
 /* Fault-path tunables: max_claims = pages one warp claims per fault round
@@ -321,7 +327,8 @@ typedef struct {
     const uint32_t* ids_dev;     /* [L][N] record ids, ascending per bucket        */
     uint64_t N;                  /* records in the file                            */
     uint32_t rec_stride;         /* bytes between records (4096 = padded, 3072)   */
-    uint32_t group;              /* candidates per warp iteration: 1, 2, 4 or 8    */
+    uint32_t group;              /* candidates per warp iteration: 1, 2, 4, 8, 16  *
+                                  * or 32 (32 / group lanes read each record)      */
     uint64_t block_begin;        /* first query block (row-major 32x32 blocks)     */
     uint64_t block_count;        /* number of query blocks                        */
     int32_t mode;                /* AP_MODE_APOINTER | AP_MODE_RAW                 */

@@ -123,6 +123,10 @@ constexpr int ERR_PERM = -9;
 
 constexpr int POLICY_CLOCK = 0;
 constexpr int POLICY_RANDOM = 1;
+/* clock + drop-behind: a warp that faults right after leaving a page first
+ * tries to reuse that page's frame (single-pass streams, like
+ * MADV_SEQUENTIAL; R-A11 leaves the policy open) */
+constexpr int POLICY_SEQUENTIAL = 2;
 
 /* Counters, sharded by SM to keep atomics off one address. */
 struct alignas(64) dev_stats {
@@ -446,7 +450,7 @@ __device__ __forceinline__ int nth_set(unsigned m, int k) {
  * S10 unlink: lanes with `mine` drop their link to
  * `page` of `r`.  Warp-aggregated: one release-add of -n per distinct page. */
 static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const dev_region* r,
-                                          uint64_t page) {
+                                          uint64_t page, bool fenced = false) {
     unsigned long long key = mine ? (((unsigned long long)r->id << 48) | page) : ~0ull;
     unsigned grp = __match_any_sync(m, key);
     unsigned lane = lane_id();
@@ -465,7 +469,11 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
                 atomicCAS(r->cache->err, 0, (o >> 62) != 2 ? -107 : -108);
         }
 #else
-        red_unlink(AP_PTE_AT(r, page), (uint64_t)0 - (uint64_t)n);
+        /* fenced: the caller issued fence.acq_rel after its last access, so a
+         * relaxed add is the release pattern of the PTX model */
+        if (fenced) red_add_relaxed(reinterpret_cast<unsigned long long*>(AP_PTE_AT(r, page)),
+                                    (unsigned long long)(0 - (uint64_t)n));
+        else red_unlink(AP_PTE_AT(r, page), (uint64_t)0 - (uint64_t)n);
 #endif
 #if defined(AP_COUNT_UNLINKS) && !defined(AP_NO_HOT_STATS)
         /* opt-in: one more atomic per unlink cost a third of the minor-fault
@@ -516,7 +524,7 @@ __device__ __forceinline__ void writeback_page(unsigned m, const dev_cache* c, c
  * victim is claimed by CAS of its PTE (VALID, rc=0) -> EMPTY, which a
  * concurrent minor fault's CAS either precedes or loses to. */
 __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, bool want,
-                                             uint32_t& frame) {
+                                             uint32_t& frame, uint32_t hint = 0) {
     const unsigned lane = lane_id();
     const int first = __ffs(m) - 1;
     const unsigned wantm = __ballot_sync(m, want);
@@ -536,20 +544,44 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         }
     }
     unsigned still = __ballot_sync(m, want && !got);
+    unsigned long long evicted = 0;
+    if (still && c->policy == POLICY_SEQUENTIAL) {
+        /* drop-behind: the frame of the page this lane's group just left
+         * (hint = frame + 1), if no pointer re-linked it meanwhile */
+        if (want && !got && hint) {
+            const uint32_t f = hint - 1;
+            const uint64_t own = f < c->frames ? ld_relaxed(c->owner + f) : 0;
+            if (own) {
+                const dev_region* vr = c->regions + ((own >> 48) - 1);
+                uint64_t* q = AP_PTE_FIND(vr, own & PAGE_MASK48);
+#ifdef AP_PT_HASH
+                const uint64_t e = q ? ld_relaxed(q) : 0;
+#else
+                const uint64_t e = ld_relaxed(q);
+#endif
+                if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f && (e & PTE_RC_MASK) == 0 &&
+                    !(e & PTE_DIRTY) && pte_cas_acquire(vr->shared, q, e, PTE_EMPTY) == e) {
+                    frame = f;
+                    got = true;
+                    ++evicted;
+                }
+            }
+        }
+        still = __ballot_sync(m, want && !got);
+    }
     /* the lanes present (possibly fewer than 32) each examine one frame per
      * clock step; at most two laps per attempt (second chance), then back off */
     const unsigned nl = __popc(m);
     const unsigned rk = __popc(m & lanemask_lt());
     const uint64_t lap = (c->frames + nl - 1) / nl;
     uint32_t steps = c->sweep_steps < 2 * lap + 1 ? c->sweep_steps : (uint32_t)(2 * lap + 1);
-    unsigned long long evicted = 0;
     while (still && steps--) {
         unsigned long long hb = 0;
         if ((int)lane == first)
-            hb = fetch_add_relaxed(c->clock_hand, c->policy == POLICY_CLOCK ? (unsigned long long)nl : 1ull);
+            hb = fetch_add_relaxed(c->clock_hand, c->policy != POLICY_RANDOM ? (unsigned long long)nl : 1ull);
         hb = __shfl_sync(m, hb, first);
         uint64_t f;
-        if (c->policy == POLICY_CLOCK) f = (hb + rk) % c->frames;
+        if (c->policy != POLICY_RANDOM) f = (hb + rk) % c->frames;
         else f = sm64(c->policy_seed ^ (hb << 5) ^ rk) % c->frames;
         bool elig = false;
         uint64_t e = 0;
@@ -565,7 +597,7 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
             e = ld_relaxed(q);
 #endif
             if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f && (e & PTE_RC_MASK) == 0) {
-                if (c->policy == POLICY_CLOCK && (e & PTE_REF)) cas_relaxed(q, e, e & ~PTE_REF);
+                if (c->policy != POLICY_RANDOM && (e & PTE_REF)) cas_relaxed(q, e, e & ~PTE_REF);
                 else elig = true;
             }
         }
@@ -709,7 +741,7 @@ struct slow_out {
  * value at the lane's offset for lanes that were unlinked. */
 template <class T>
 __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t page,
-                                               const dev_region* r) {
+                                               const dev_region* r, uint32_t hint = 0) {
     /* Lanes linked on entry reload their value here, so the caller's
      * speculative load is dead on this path and is never kept live across
      * the call (keeping it live made every hit-path load wait for its data
@@ -793,7 +825,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         /* Phase B: frames for the claimed pages (S7). */
         const unsigned claimed = __ballot_sync(m, st == ST_CLAIMED);
         if (claimed) {
-            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame);
+            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame, hint);
             if (st == ST_CLAIMED && !ok) {
                 /* give the page back (an add, so transient counts survive) */
                 pte_red_release(r->shared, pte, (uint64_t)0 - PTE_LOADING);
@@ -1233,12 +1265,12 @@ struct ptr {
      * (warp-aggregated), then unlinked lanes link -- inline when the page is
      * resident (link_minor), else through the fault handler. */
     __device__ __forceinline__ T deref_miss(unsigned m) {
-        drop_stale(m);
+        const uint32_t hint = drop_stale(m);
         if (detail::try_link_minor<T>(m, x, page, r, lg)) {
             sync_fb();
             return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
         }
-        const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
+        const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r, hint);
         x = o.x;
         page = o.page;
         sync_fb();
@@ -1473,6 +1505,24 @@ struct ptr {
         return *(volatile unsigned long long*)c->free_head >= c->nfree;
     }
 
+    /* Unlink after an explicit ap::fence_acq_rel() that follows the last
+     * access through the pointer (the fence + relaxed add is the release
+     * pattern of the PTX memory model): lets one fence serve several
+     * pointers -- and, after a link_begin, also the acquire of that link
+     * (relaxed add observed, then the fence). */
+    __device__ __forceinline__ void release_fenced() {
+        const unsigned m = __activemask();
+        const bool l = holds();
+        if (__any_sync(m, l)) {
+            const uint64_t off = foff();
+            detail::unlink_lanes(m, l, r, page, true);
+            if (l) {
+                x = off;
+                fb = XL_VALID;
+            }
+        }
+    }
+
     /* Unlink now (also done by the destructor and by assignment). */
     __device__ __forceinline__ void release() {
         const unsigned m = __activemask();
@@ -1494,22 +1544,25 @@ struct ptr {
     }
     /* lanes that walked off their frame unlink it and carry
      * on unlinked at the same file offset */
-    __device__ __forceinline__ void drop_stale(unsigned m) {
+    __device__ __forceinline__ uint32_t drop_stale(unsigned m) {
         const bool stale = holds() && !ready();
+        uint32_t hint = 0; /* the dropped frame + 1 (drop-behind policy) */
         if (__any_sync(m, stale)) {
             const uint64_t off = foff();
+            if (stale) hint = (uint32_t)((((fb & XL_ADDR) - (uint64_t)r->pool) >> lg) + 1);
             detail::unlink_lanes(m, stale, r, page);
             if (stale) {
                 x = off;
                 fb = XL_VALID;
             }
         }
+        return hint;
     }
     /* make every lane of m linked at its current offset */
     __device__ __forceinline__ void relink(unsigned m) {
-        drop_stale(m);
+        const uint32_t hint = drop_stale(m);
         if (__any_sync(m, !holds()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
-            const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r);
+            const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r, hint);
             x = o.x;
             page = o.page;
         }
@@ -1521,6 +1574,9 @@ struct ptr {
         fb = XL_VALID;
     }
 };
+
+/* A GPU-scope acq_rel fence (see ptr::release_fenced, ptr::link_finish). */
+__device__ __forceinline__ void fence_acq_rel() { detail::fence_gpu(); }
 
 /* gvmmap (M17): an unlinked apointer to byte offset
  * `foff` of region `region` of the cache.  Read-only mappings only. */

@@ -12,7 +12,7 @@ LIB_PATH = os.environ.get("AP_LIB_PATH") or os.path.join(_HERE, "libapointer.so"
 AP_OK = 0
 AP_EINVAL, AP_ENOMEM, AP_ECUDA, AP_EBUSY, AP_ERANGE = -1, -2, -3, -4, -5
 AP_EFAULT, AP_ENOFRAME, AP_ETIMEDOUT = -6, -7, -8
-AP_POLICY_CLOCK, AP_POLICY_RANDOM = 0, 1
+AP_POLICY_CLOCK, AP_POLICY_RANDOM, AP_POLICY_SEQUENTIAL = 0, 1, 2
 AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
 AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_AHEAD, AP_ACCESS_PAIR, AP_ACCESS_TMA = 0, 1, 2, 3, 4, 5

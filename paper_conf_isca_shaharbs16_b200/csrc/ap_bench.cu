@@ -332,13 +332,18 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
     const uint32_t per_unit = a.unit / (32 * E);
     uint64_t h = FNV_BASIS;
+    /* one pointer per thread walks its units: moving it to the next unit is
+     * arithmetic, and the page it leaves is unlinked by the next unit's first
+     * dereference (which can then reuse that frame, AP_POLICY_SEQUENTIAL) */
+    [[maybe_unused]] ap::ptr<T> q;
+    if constexpr (APTR) q = ap::gvmmap<T>(c, region, 0);
     for (uint32_t pass = 0; pass < a.passes; ++pass) {
         for (uint64_t u = w; u < nunits; u += W) {
             const uint64_t e0 = u * (a.unit / E) + lane;
             /* whole unit inside the span: tiled fast loop; else per element */
             const bool whole = (u + 1) * a.unit <= a.span;
             if constexpr (APTR) {
-                ap::ptr<T> q = ap::gvmmap<T>(c, region, e0 * E);
+                q += (int64_t)(e0 * E - q.foff()) / (int64_t)E;
                 if (a.access == AP_ACCESS_RANGE && whole) {
                     /* translate once for the unit, then stream plain loads
                      * through the linked translation (valid while q lives) */

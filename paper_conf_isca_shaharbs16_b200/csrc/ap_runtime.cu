@@ -762,7 +762,9 @@ extern "C" int ap_cache_reset(ap_cache_t c) {
 }
 
 extern "C" int ap_cache_set_policy(ap_cache_t c, int policy, uint64_t seed) {
-    if (!c || (policy != AP_POLICY_CLOCK && policy != AP_POLICY_RANDOM)) return AP_EINVAL;
+    if (!c || (policy != AP_POLICY_CLOCK && policy != AP_POLICY_RANDOM &&
+               policy != AP_POLICY_SEQUENTIAL))
+        return AP_EINVAL;
     ap_device_guard g(c->device);
     AP_CUDA_TRY(cudaDeviceSynchronize());
     c->h.policy = policy;

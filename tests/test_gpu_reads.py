@@ -352,3 +352,34 @@ def test_link_events_closed_form(ap, dev, pattern, elem, page, nbytes, prefill):
         ap.ap_munmap(cache, r)
     finally:
         ap.ap_cache_destroy(cache)
+
+
+@pytest.mark.parametrize("frames", [1, 3, 64, 4096])
+@pytest.mark.parametrize("pattern", ["seq", "uniform"])
+def test_sequential_policy_drop_behind(ap, dev, frames, pattern):
+    """AP_POLICY_SEQUENTIAL (the clock + drop-behind: a faulting warp first
+    reuses the frame of the page it just left): values are the file's bytes
+    under any order of eviction, invariants hold, and a
+    single-pass stream through few frames recycles frames without sweeping."""
+    nbytes = (1 << 20) + 5 * 4096 + 32
+    f = make_file(nbytes, seed=91)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        ap.ap_cache_set_policy(cache, ap.AP_POLICY_SEQUENTIAL)
+        r = ap.ap_mmap(cache, f)
+        if pattern == "seq":
+            grid, block = (2, 64) if frames < 8 else (8, 128)
+            cfg = ap.bench_cfg(ap.AP_SEQ, 16, grid, block, unit_bytes=4096, out_copy=True,
+                               span_bytes=nbytes)
+            out = _run(ap, cache, r, cfg, grid * block, dev, out_bytes=nbytes)
+            whole = nbytes // 16 * 16
+            assert np.array_equal(out[:whole], f[:whole])
+        else:
+            grid, block, reads = 6, 128, 5
+            cfg = ap.bench_cfg(ap.AP_UNIFORM, 4, grid, block, reads_per_thread=reads, seed=19)
+            got = _run(ap, cache, r, cfg, grid * block, dev).view(np.uint64)
+            assert np.array_equal(got, oracle.read_uniform(f, nbytes, 4, grid * block, reads, 19))
+        assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        ap.ap_cache_destroy(cache)
