@@ -1,24 +1,41 @@
 """profiles/traffic.json from the ncu --set full summaries in profiles/ (DRAM
-read + write bytes per launch of each dominant kernel)."""
+read + write bytes per launch of each dominant kernel; every summary names
+its kernels in capture order: apointer first, then the raw twin)."""
 import json
 import re
+import sys
+
+R = sys.argv[1] if len(sys.argv) > 1 else "r02"
 
 
-def first_bytes(path, idx=0):
+def kernel_bytes(path):
+    """[(kernel line, dram read + write bytes)] in the order of the report."""
     t = open(path).read()
+    names = [m for m in re.findall(r"^(.*?) \| Duration", t, re.M)]
     rd = re.findall(r'raw dram__bytes_read.sum = ([0-9.]+) (\w+)', t)
     wr = re.findall(r'raw dram__bytes_write.sum = ([0-9.]+) (\w+)', t)
     mul = {'byte': 1, 'Kbyte': 1e3, 'Mbyte': 1e6, 'Gbyte': 1e9}
-    return float(rd[idx][0]) * mul[rd[idx][1]] + float(wr[idx][0]) * mul[wr[idx][1]]
+    return [(n, float(a[0]) * mul[a[1]] + float(b[0]) * mul[b[1]]) for n, a, b in zip(names, rd, wr)]
+
+
+def entry(path, idx, what):
+    ks = kernel_bytes(path)
+    name, b = ks[idx]
+    return {"dram_bytes_per_launch": b, "kernel_in_capture": name.strip(),
+            "source": f"{path} (ncu --set full; {what})"}
 
 
 tj = {
-    "k_random<uint32_t, UNIFORM, apointer>": {"dram_bytes_per_launch": first_bytes('profiles/r01_full_c2.txt'), "source": "profiles/r01_full_c2.txt (ncu --set full, 1 launch; DRAM read + write: the frame fills are the writes)"},
-    "k_seq<uint4, apointer>": {"dram_bytes_per_launch": first_bytes('profiles/r01_full_hit.txt'), "source": "profiles/r01_full_hit.txt (ncu --set full, 1 launch, 2 passes over 1 GiB)"},
-    "k_seq<uint4, raw>": {"dram_bytes_per_launch": first_bytes('profiles/r01_full_hit_raw.txt'), "source": "profiles/r01_full_hit_raw.txt (ncu --set full, 1 launch, 2 passes over 1 GiB)"},
-    "k_collage<8, apointer>": {"dram_bytes_per_launch": first_bytes('profiles/r01_full_c4.txt'), "source": "profiles/r01_full_c4.txt (ncu --set full, 1 launch = one of the 12 record-id window passes of a cold C4 step)"},
-    "k_collage<8, apointer> resident": {"dram_bytes_per_launch": first_bytes('profiles/r01_full_c4_resident.txt', 1), "source": "profiles/r01_full_c4_resident.txt (second kernel: the resident-cache run; the first is the cold run that fills the cache)"},
-    "k_random<uint32_t, UNIFORM, apointer> resident (M2r)": {"dram_bytes_per_launch": first_bytes('profiles/r01_full_minor.txt'), "source": "profiles/r01_full_minor.txt (ncu --set full; first launch = apointer, second = raw twin)"},
+    "k_random<uint32_t, UNIFORM, apointer>": entry(f"profiles/{R}_full_c2.txt", 0, "one C2 launch, cold cache: the frame fills are the writes"),
+    "k_seq<uint4, apointer>": entry(f"profiles/{R}_full_k_seq.txt", 0, "tile hit mode, 2 passes over 1 GiB"),
+    "k_seq<uint4, raw>": entry(f"profiles/{R}_full_k_seq.txt", 1, "raw twin of the same launch"),
+    "k_seq_deref<uint4, apointer>": entry(f"profiles/{R}_full_k_seq_deref.txt", 0, "per-access form, 2 passes over 1 GiB"),
+    "k_seq_deref<uint4, raw>": entry(f"profiles/{R}_full_k_seq_deref.txt", 1, "raw twin of the same launch"),
+    "k_random<uint32_t, UNIFORM, apointer> resident (M2r)": entry(f"profiles/{R}_full_k_random.txt", 0, "M2r: uniform 4-B reads over the resident GiB"),
+    "k_random<uint32_t, UNIFORM, raw> resident (M2r)": entry(f"profiles/{R}_full_k_random.txt", 1, "the raw gather twin"),
+    "k_collage<8, apointer>": entry(f"profiles/{R}_full_c4.txt", 0, "one launch = one of the 12 record-id window passes of a cold C4 step"),
+    "k_collage<8, apointer> resident": entry(f"profiles/{R}_full_c4_resident.txt", 0, "cache holds every record"),
+    "k_collage<8, raw> resident": entry(f"profiles/{R}_full_c4_resident.txt", 1, "raw twin on an HBM copy"),
 }
 json.dump(tj, open('profiles/traffic.json', 'w'), indent=1)
-print(json.dumps({k: v["dram_bytes_per_launch"] for k, v in tj.items()}, indent=1))
+print(json.dumps({k: (v["dram_bytes_per_launch"], v["kernel_in_capture"][:50]) for k, v in tj.items()}, indent=1))

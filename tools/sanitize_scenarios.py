@@ -175,5 +175,50 @@ ap.ap_munmap(ca, ra)
 ap.ap_munmap(cb, rb)
 ap.ap_cache_destroy(ca)
 ap.ap_cache_destroy(cb)
+
+# [r2] per-access dereference (deferred unlink at the next dereference) and the
+# drop-behind policy, with frames scarce; Fig. 6 ADD (two pointers, the miss
+# path releases the other one under pressure)
+fd_ = make_file((1 << 20) + 4096 * 3 + 48, 2)
+for frames, policy in ((3, ap.AP_POLICY_SEQUENTIAL), (5, ap.AP_POLICY_CLOCK)):
+    c = ap.ap_cache_create(frames, 4096)
+    ap.ap_cache_set_policy(c, policy)
+    r = ap.ap_mmap(c, fd_)
+    ck = torch.zeros(128, dtype=torch.int64, device=dev)
+    ap.ap_bench_read(c, r, ap.bench_cfg(ap.AP_SEQ, 16, 1, 128, unit_bytes=4096,
+                                        access=ap.AP_ACCESS_DEREF), ck)
+    torch.cuda.synchronize()
+    check(f"deref frames={frames} policy={policy}", np.array_equal(
+XX, check_invariants(ap, c, [r], frames) == [])
+    ap.ap_munmap(c, r)
+    ap.ap_cache_destroy(c)
+fa = make_file(1 << 21, 4)
+c = ap.ap_cache_create(4, 4096)
+r = ap.ap_mmap(c, fa)
+acc = torch.zeros(64, dtype=torch.int64, device=dev)
+ap.ap_bench_compute(c, r, "add", 16, 1, 64, 1 << 20, acc)
+torch.cuda.synchronize()
+want = oracle.compute(fa, 1 << 20, 4096, 16, 64, 0)
+check("compute add frames=4", np.array_equal(acc.cpu().numpy().view(np.uint64).astype(np.float64),
+                                              want))
+check("compute add invariants", check_invariants(ap, c, [r], 4) == [])
+ap.ap_munmap(c, r)
+ap.ap_cache_destroy(c)
+
+# [r2] multi-partition collage through the C ABI (three partitions on this
+# GPU fold winners into one array with system-scope atomics)
+nm = 600
+recs_m = make_records(nm, 4096, 13)
+proj_m, bias_m = synth.make_lsh_params(2, 4, 2500, seed=14)
+img_m, _, _ = synth.make_target(128, 64, nm, ds_seed=13, seed=15, pool=8, copy_permille=100)
+o_off_m, o_ids_m = oracle.build_index(recs_m, 4096, nm, proj_m, bias_m, 2500, 6)
+want_m = oracle.collage(img_m, proj_m, bias_m, 2500, 6, recs_m, 4096, nm, o_off_m, o_ids_m)
+for part in (ap.AP_PART_BLOCKS, ap.AP_PART_RECORDS):
+    win_m = np.zeros(((128 // 32) * (64 // 32), 2), dtype=np.uint32)
+    inp_m = ap.mgpu_collage_in(img_m, 128, 64, proj_m, bias_m, 2500, 6, nm, group=4,
+                               partition=part)
+    rep = ap.ap_collage_mgpu([0, 0, 0], recs_m, 5, 4096, inp_m, win_m)
+    check(f"mgpu partition={part}", np.array_equal(win_m, want_m) and rep["device_error"] == 0)
+
 print("ALL OK" if ok else "FAILURES")
 sys.exit(0 if ok else 1)
