@@ -23,7 +23,8 @@ CFLAGS  := -O2 -fopenmp -fPIC -Wall -Wextra -std=c11
 CU_SRCS := $(wildcard $(CSRC)/*.cu)
 CU_HDRS := $(wildcard $(CSRC)/*.cuh) $(wildcard include/*.h) $(wildcard include/ap/*.cuh)
 
-all: synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so $(PKG)/libapointer_hash.so
+all: synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so $(PKG)/libapointer_hash.so \
+     tools/atomic_ceiling
 
 synth/libsynth.so: synth/synth.c
 	$(HOSTCC) $(CFLAGS) -shared $< -o $@ -lm
@@ -38,12 +39,17 @@ $(PKG)/libapointer.so: $(CU_SRCS) $(CU_HDRS)
 $(PKG)/libapointer_hash.so: $(CU_SRCS) $(CU_HDRS)
 	$(NVCC) $(NVFLAGS) -DAP_PT_HASH -shared $(CU_SRCS) -o $@ -lcuda
 
+# the M2r ceiling (bench.py runs it in the same session as the kernels it bounds)
+tools/atomic_ceiling: tools/atomic_ceiling.cu
+	$(NVCC) -O3 $(ARCH) $< -o $@
+
 host: synth/libsynth.so oracle/liboracle.so
 
 sass: $(PKG)/libapointer.so
 	/usr/local/cuda/bin/cuobjdump -sass $< > build_sass.txt
 
 clean:
-	rm -f synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so $(PKG)/libapointer_hash.so
+	rm -f synth/libsynth.so oracle/liboracle.so $(PKG)/libapointer.so $(PKG)/libapointer_hash.so \
+	      tools/atomic_ceiling
 
 .PHONY: all host clean sass

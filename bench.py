@@ -331,10 +331,32 @@ def run_hit(args, torch, dev, ap, cache, region, f, stream, span=GiB, passes=8):
         majors=st_m1["major"] - st_m0["major"],
         minors_per_launch=(st_m1["minor"] - st_m0["minor"]) / max(1, len(t_m) + max(args.warmup, 3)),
         equal_raw=bool(torch.equal(out_m, out_mr)), grid=grid_m)
+    # the M2r ceiling, measured here: the same memory operations per read (an
+    # acquire add and a release add on random entries of a 16 384-entry PTE
+    # array + the 4-B gather) with no page-cache logic (tools/atomic_ceiling.cu)
+    res["minor"]["ceiling"] = m2r_ceiling()
     del dcopy
     res.update(majors_during=st1["major"] - st0["major"], checksums_equal_raw=same,
                ap_gbs=res["tile"]["gbs"], overhead=res["tile"]["overhead"])
     return res
+
+
+def m2r_ceiling():
+    """G steps/s of tools/atomic_ceiling (built by make), or None."""
+    exe = os.path.join(ROOT, "tools", "atomic_ceiling")
+    if not os.path.exists(exe):
+        return None
+    try:
+        out = subprocess.run([exe], capture_output=True, text=True, timeout=120).stdout
+    except Exception:
+        return None
+    import re
+    res = {}
+    for line in out.splitlines():
+        m = re.match(r"^(.*?)\s+([0-9.]+) G steps/s", line)
+        if m:
+            res[m.group(1).strip()] = float(m.group(2)) * 1e9
+    return res or None
 
 
 def cpu_oracle_c2(res, threads):
@@ -459,6 +481,16 @@ def emit_c2(args, res_all, rank, world):
             "useful_GBps": round(hit["minor"]["useful_gbs"], 3),
             "sector_GBps": round(hit["minor"]["sector_gbs"], 3),
             "overhead_vs_raw": round(hit["minor"]["overhead"], 4),
+            "ceiling_reads_per_s": (hit["minor"]["ceiling"] or {}).get(
+                "acquire add + 4-B gather + release add"),
+            "frac_of_ceiling": (round(hit["minor"]["reads_per_s"] /
+                                      hit["minor"]["ceiling"]["acquire add + 4-B gather + release add"], 4)
+                                if hit["minor"].get("ceiling") else None),
+            "ceiling_note": "tools/atomic_ceiling, run in this session: per read one acquire add "
+                            "and one release add on random entries of a 16 384-entry PTE array "
+                            "plus the 4-B gather, no page-cache logic (all G steps/s: "
+                            "%s)" % {k: round(v / 1e9, 2) for k, v in
+                                     (hit["minor"].get("ceiling") or {}).items()},
             "major_faults_during": hit["minor"]["majors"],
             "minor_faults_per_launch": hit["minor"]["minors_per_launch"],
             "checksums_equal_raw": hit["minor"]["equal_raw"]},

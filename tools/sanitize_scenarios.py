@@ -189,7 +189,8 @@ for frames, policy in ((3, ap.AP_POLICY_SEQUENTIAL), (5, ap.AP_POLICY_CLOCK)):
                                         access=ap.AP_ACCESS_DEREF), ck)
     torch.cuda.synchronize()
     check(f"deref frames={frames} policy={policy}", np.array_equal(
-XX, check_invariants(ap, c, [r], frames) == [])
+        ck.cpu().numpy().view(np.uint64), oracle.read_seq(fd_, fd_.nbytes, 4096, 16, 128, 1)))
+    check(f"deref invariants frames={frames}", check_invariants(ap, c, [r], frames) == [])
     ap.ap_munmap(c, r)
     ap.ap_cache_destroy(c)
 fa = make_file(1 << 21, 4)
