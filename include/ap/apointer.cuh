@@ -524,7 +524,9 @@ __device__ __forceinline__ void writeback_page(unsigned m, const dev_cache* c, c
  * victim is claimed by CAS of its PTE (VALID, rc=0) -> EMPTY, which a
  * concurrent minor fault's CAS either precedes or loses to. */
 __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, bool want,
-                                             uint32_t& frame, uint32_t hint = 0) {
+                                             uint32_t& frame, uint32_t hint = 0,
+                                             const dev_region* hint_r = nullptr,
+                                             uint64_t hint_page = 0) {
     const unsigned lane = lane_id();
     const int first = __ffs(m) - 1;
     const unsigned wantm = __ballot_sync(m, want);
@@ -548,21 +550,23 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
     if (still && c->policy == POLICY_SEQUENTIAL) {
         /* drop-behind: the frame of the page this lane's group just left
          * (hint = frame + 1), if no pointer re-linked it meanwhile */
-        if (want && !got && hint) {
+        if (want && !got && hint && hint_r) {
+            /* the left page's entry is known (no owner-table lookup): try
+             * the CAS against its expected value (VALID, this frame,
+             * referenced, count 0), then once against what it holds */
             const uint32_t f = hint - 1;
-            const uint64_t own = f < c->frames ? ld_relaxed(c->owner + f) : 0;
-            if (own) {
-                const dev_region* vr = c->regions + ((own >> 48) - 1);
-                uint64_t* q = AP_PTE_FIND(vr, own & PAGE_MASK48);
-#ifdef AP_PT_HASH
-                const uint64_t e = q ? ld_relaxed(q) : 0;
-#else
-                const uint64_t e = ld_relaxed(q);
-#endif
-                if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f && (e & PTE_RC_MASK) == 0 &&
-                    !(e & PTE_DIRTY) && pte_cas_acquire(vr->shared, q, e, PTE_EMPTY) == e) {
-                    frame = f;
+            uint64_t* q = AP_PTE_FIND(hint_r, hint_page);
+            if (f < c->frames && q) {
+                const uint64_t want_e = PTE_VALID | PTE_REF | ((uint64_t)f << 32);
+                uint64_t e = pte_cas_acquire(hint_r->shared, q, want_e, PTE_EMPTY);
+                if (e == want_e) {
                     got = true;
+                } else if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f &&
+                           (e & PTE_RC_MASK) == 0 && !(e & PTE_DIRTY)) {
+                    got = pte_cas_acquire(hint_r->shared, q, e, PTE_EMPTY) == e;
+                }
+                if (got) {
+                    frame = f;
                     ++evicted;
                 }
             }
@@ -739,9 +743,16 @@ struct slow_out {
  * Called by the converged lanes `m` when at least one of them is unlinked.
  * Returns each lane's new translation and linked page; `val` receives the
  * value at the lane's offset for lanes that were unlinked. */
+/* hint (optional, per lane): bit 31 = the inline link just found this
+ * lane's page EMPTY (the first round claims it without probing again); bits
+ * 30:0 = frame + 1 of the page the lane's pointer left just before (hint_page
+ * of the same region), for the drop-behind policy. */
 template <class T>
 __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t page,
-                                               const dev_region* r, uint32_t hint = 0) {
+                                               const dev_region* r, uint32_t hint = 0,
+                                               uint64_t hint_page = 0) {
+    bool absent = (hint >> 31) != 0;
+    hint &= 0x7fffffffu;
     /* Lanes linked on entry reload their value here, so the caller's
      * speculative load is dead on this path and is never kept live across
      * the call (keeping it live made every hit-path load wait for its data
@@ -790,7 +801,12 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
          * add is undone.  Every other transition tolerates such transient
          * counts on non-VALID entries: publish and revert are adds, claims
          * are CASes from exactly EMPTY (R-A17). */
-        uint64_t old = is_leader ? add_link(pte, n) : 0;
+        /* first round after an inline link found the page EMPTY: go straight
+         * to the claim (a race with a concurrent claim or publish just makes
+         * the CAS fail and the next round probe again) */
+        const bool probed = is_leader && !absent;
+        uint64_t old = probed ? add_link(pte, n) : 0;
+        absent = false;
 #ifdef AP_DEBUG
         if (is_leader && (old >> 62) == 2) printf("[link] w%u m%08x n%u pg %llu old %llx\n", (unsigned)(threadIdx.x >> 5), m, n, (unsigned long long)pg, (unsigned long long)old);
 #endif
@@ -799,7 +815,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
                 st = ST_LINKED;
                 frame = (uint32_t)((old >> 32) & PTE_FRAME_MASK);
                 if (!(old & PTE_REF)) red_or_relaxed(pte, PTE_REF);
-            } else {
+            } else if (probed) {
                 red_add_relaxed(reinterpret_cast<unsigned long long*>(pte),
                                 (unsigned long long)(0 - (uint64_t)n));
             }
@@ -825,7 +841,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         /* Phase B: frames for the claimed pages (S7). */
         const unsigned claimed = __ballot_sync(m, st == ST_CLAIMED);
         if (claimed) {
-            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame, hint);
+            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame, hint, r, hint_page);
             if (st == ST_CLAIMED && !ok) {
                 /* give the page back (an add, so transient counts survive) */
                 pte_red_release(r->shared, pte, (uint64_t)0 - PTE_LOADING);
@@ -945,7 +961,8 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
  * case no register state is saved around an out-of-line call. */
 template <class T>
 __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& page,
-                                           const dev_region* r, uint32_t lg) {
+                                           const dev_region* r, uint32_t lg,
+                                           uint32_t* absent = nullptr) {
     const bool need = !(x >> 63);
     /* out-of-range / misaligned offsets: the full path reports them */
     if (__any_sync(m, need && (x + sizeof(T) > r->bytes || (x % sizeof(T)) != 0))) return false;
@@ -985,6 +1002,8 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
         x = XL_VALID | ((uint64_t)(r->pool + f * P) + (x & (P - 1)));
         page = pg;
     }
+    /* the page was not resident (EMPTY): the fault path may claim it at once */
+    if (absent) *absent = (need && (old >> 62) == 0) ? 1u : 0u;
     return __all_sync(m, ok);
 }
 
@@ -992,11 +1011,13 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
  * through the out-of-line fault path) */
 template <class T>
 __device__ __forceinline__ bool try_link_minor(unsigned m, uint64_t& x, uint64_t& page,
-                                               const dev_region* r, uint32_t lg) {
+                                               const dev_region* r, uint32_t lg,
+                                               uint32_t* absent = nullptr) {
 #ifdef AP_NO_LINK_MINOR
+    if (absent) *absent = 0;
     return false;
 #else
-    return link_minor<T>(m, x, page, r, lg);
+    return link_minor<T>(m, x, page, r, lg, absent);
 #endif
 }
 
@@ -1265,12 +1286,15 @@ struct ptr {
      * (warp-aggregated), then unlinked lanes link -- inline when the page is
      * resident (link_minor), else through the fault handler. */
     __device__ __forceinline__ T deref_miss(unsigned m) {
+        const uint64_t left = page;
         const uint32_t hint = drop_stale(m);
-        if (detail::try_link_minor<T>(m, x, page, r, lg)) {
+        uint32_t absent = 0;
+        if (detail::try_link_minor<T>(m, x, page, r, lg, &absent)) {
             sync_fb();
             return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
         }
-        const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r, hint);
+        const detail::slow_out<T> o =
+            detail::deref_slow<T>(m, x, page, r, hint | (absent << 31), left);
         x = o.x;
         page = o.page;
         sync_fb();
@@ -1560,9 +1584,12 @@ struct ptr {
     }
     /* make every lane of m linked at its current offset */
     __device__ __forceinline__ void relink(unsigned m) {
+        const uint64_t left = page;
         const uint32_t hint = drop_stale(m);
-        if (__any_sync(m, !holds()) && !detail::try_link_minor<T>(m, x, page, r, lg)) {
-            const detail::slow_out<T> o = detail::deref_slow<T>(m, x, page, r, hint);
+        uint32_t absent = 0;
+        if (__any_sync(m, !holds()) && !detail::try_link_minor<T>(m, x, page, r, lg, &absent)) {
+            const detail::slow_out<T> o =
+                detail::deref_slow<T>(m, x, page, r, hint | (absent << 31), left);
             x = o.x;
             page = o.page;
         }

@@ -137,8 +137,16 @@ def test_hit_mode_after_prefill_has_no_major_faults(ap, dev):
         assert np.array_equal(got, want)
         st1 = ap.ap_cache_stats(cache)
         assert st1["major"] == st0["major"]
-        # one link per (warp, unit) visit: SEQ with unit | page, all lanes on one page
-        assert st1["minor"] - st0["minor"] == 2 * (nbytes // 16384)
+        # SEQ with unit | page, all lanes of a warp on one page, one pointer per
+        # thread walking its units: one link each time the warp's next unit is
+        # on another page than the one it holds -- a warp whose
+        # only unit is revisited by the next pass keeps its link
+        W, nunits, upp = grid * block // 32, nbytes // 16384, page // 16384
+        links = 0
+        for w in range(W):
+            pages = [u // upp for _ in range(2) for u in range(w, nunits, W)]
+            links += sum(1 for i, p in enumerate(pages) if i == 0 or p != pages[i - 1])
+        assert st1["minor"] - st0["minor"] == links
         assert check_invariants(ap, cache, [r], frames) == []
         # raw twin over an HBM copy reads the same values
         dcopy = torch.from_numpy(f).to(dev)

@@ -1,0 +1,10 @@
+#!/bin/bash
+# round 2 pass 14: suite on the fault-path latency changes (no second probe
+# after an inline link found the page EMPTY; drop-behind CAS on the left
+# page's known entry), C1/C2/C3 lines
+mkdir -p gpurun_out
+timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/r2_tests14.txt 2>&1
+echo "rc=$?" >> gpurun_out/r2_tests14.txt
+python bench.py --workload c1 --steps 5 --warmup 3 > gpurun_out/r2_bench_c1.json 2> gpurun_out/r2_bench_c1.err
+python bench.py --workload c3 --steps 3 --warmup 2 --no-cpu-baseline > gpurun_out/r2_bench_c3.json 2> gpurun_out/r2_bench_c3.err
+python bench.py --steps 5 --warmup 3 > gpurun_out/r2_bench_default.json 2> gpurun_out/r2_bench_default.err
