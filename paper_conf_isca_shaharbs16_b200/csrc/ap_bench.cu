@@ -567,6 +567,13 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
     a->span = cfg->span_bytes ? cfg->span_bytes : rg.bytes;
     a->access = cfg->access;
     if (cfg->access < AP_ACCESS_TILE || cfg->access > AP_ACCESS_TMA) return AP_EINVAL;
+#ifdef AP_PT_HASH
+    /* the split-phase link styles are not part of the hash-table ablation
+     * (their relaxed early adds race with its probes) */
+    if (cfg->mode == AP_MODE_APOINTER &&
+        (cfg->access == AP_ACCESS_AHEAD || cfg->access == AP_ACCESS_PAIR))
+        return AP_EINVAL;
+#endif
     switch (cfg->pattern) {
         case AP_SEQ:
             if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;

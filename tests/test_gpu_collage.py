@@ -8,7 +8,7 @@ import torch
 
 import oracle
 import synth
-from helpers import check_invariants, make_records
+from helpers import check_invariants, make_records, teardown
 from paper_conf_isca_shaharbs16_b200 import mgpu
 
 pytestmark = pytest.mark.gpu
@@ -46,7 +46,7 @@ def test_index_matches_oracle(ap, K, bb):
         assert np.array_equal(ids.cpu().numpy().view(np.uint32), want_ids)
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1), (1, 2), (8, 2), (1, 3), (8, 3)])
@@ -89,7 +89,7 @@ def test_collage_matches_oracle(ap, group, schedule, frames):
         assert np.array_equal(win2.cpu().numpy().view(np.uint32), want)
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 def test_collage_partitioned_blocks_equal_whole(ap):
@@ -118,7 +118,7 @@ def test_collage_partitioned_blocks_equal_whole(ap):
         assert torch.equal(torch.cat(parts), full)
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("schedule", [2, 3])
@@ -162,7 +162,7 @@ def test_collage_unit_slices_min_reduce_to_whole(ap, world, schedule):
         assert check_invariants(ap, cache, [r], 90) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("group,schedule", [(1, 1), (2, 1), (4, 1), (8, 1), (4, 2), (8, 2), (8, 3)])
@@ -194,7 +194,7 @@ def test_unaligned_records_collage(ap, group, schedule, frames):
         assert check_invariants(ap, cache, [r], frames) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("schedule,chunks,frames", [(2, 2, 40), (2, 5, 40), (3, 3, 40), (3, 7, 400)])
@@ -245,7 +245,7 @@ def test_collage_record_id_windows(ap, schedule, chunks, frames):
                                                       schedule=1, id_chunks=2), win)
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("world,chunks", [(2, 0), (3, 2), (8, 1)])
@@ -297,7 +297,7 @@ def test_collage_record_slices_min_reduce_to_whole(ap, world, chunks):
                                                           **bad), part)
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("schedule", [0, 1, 2, 3])
@@ -333,4 +333,4 @@ def test_empty_candidate_sets_give_the_sentinel(ap, group, schedule):
         assert check_invariants(ap, cache, [r], 32) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)

@@ -5,7 +5,7 @@ import pytest
 import torch
 
 import oracle
-from helpers import make_file
+from helpers import make_file, teardown
 
 pytestmark = pytest.mark.gpu
 
@@ -41,4 +41,4 @@ def test_workload_parity(ap, work, elem):
             assert np.array_equal(got, want)
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)

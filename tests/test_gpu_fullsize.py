@@ -9,7 +9,7 @@ import torch
 
 import oracle
 import synth
-from helpers import aligned_empty, check_invariants, make_file
+from helpers import aligned_empty, check_invariants, make_file, teardown
 
 pytestmark = pytest.mark.gpu
 
@@ -47,7 +47,7 @@ def test_c1_full_copy(ap, dev):
         assert check_invariants(ap, cache, [r], 64) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 def test_c2_full(ap, dev):
@@ -66,7 +66,7 @@ def test_c2_full(ap, dev):
         assert check_invariants(ap, cache, [r], 16384) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 def test_c3_full(ap, dev):
@@ -84,7 +84,7 @@ def test_c3_full(ap, dev):
         assert check_invariants(ap, cache, [r], 65536) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
     del f
 
 
@@ -123,4 +123,4 @@ def test_c4_full(ap, dev, schedule):
         assert check_invariants(ap, cache, [r], 65536) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)

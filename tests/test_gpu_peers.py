@@ -16,7 +16,7 @@ import pytest
 import torch
 
 import oracle
-from helpers import check_invariants, make_file
+from helpers import check_invariants, make_file, teardown
 
 pytestmark = pytest.mark.gpu
 
@@ -69,8 +69,8 @@ def test_all_pages_from_a_full_peer(ap, dev):
         ap.ap_munmap(b, rb)
         ap.ap_munmap(a, ra)
     finally:
-        ap.ap_cache_destroy(b)
-        ap.ap_cache_destroy(a)
+        teardown(ap, b)
+        teardown(ap, a)
 
 
 def test_split_between_peer_and_host(ap, dev):
@@ -102,8 +102,8 @@ def test_split_between_peer_and_host(ap, dev):
         ap.ap_munmap(b, rb)  # clears the peer list itself
         ap.ap_munmap(a, ra)
     finally:
-        ap.ap_cache_destroy(b)
-        ap.ap_cache_destroy(a)
+        teardown(ap, b)
+        teardown(ap, a)
 
 
 @pytest.mark.parametrize("frames", [4, 48])
@@ -149,8 +149,8 @@ def test_mutual_peers_running_concurrently(ap, dev, frames):
         ap.ap_munmap(a, ra)
         ap.ap_munmap(b, rb)
     finally:
-        ap.ap_cache_destroy(a)
-        ap.ap_cache_destroy(b)
+        teardown(ap, a)
+        teardown(ap, b)
 
 
 def test_peer_argument_errors(ap, dev):
@@ -188,7 +188,7 @@ def test_peer_argument_errors(ap, dev):
             ap.ap_munmap(cache, reg)
     finally:
         for x in [a, b, c] + peers:
-            ap.ap_cache_destroy(x)
+            teardown(ap, x)
 
 
 def _ipc_exporter(q_handle, q_done, nbytes, npages):
@@ -237,7 +237,7 @@ def test_peer_in_another_process_via_ipc(ap, dev):
             ap.ap_region_clear_peers(b, rb)
             ap.ap_munmap(b, rb)
         finally:
-            ap.ap_cache_destroy(b)
+            teardown(ap, b)
         qd.put(True)
         assert qh.get(timeout=120) is True
     finally:

@@ -8,7 +8,7 @@ import pytest
 import torch
 
 import oracle
-from helpers import check_invariants, make_file
+from helpers import check_invariants, make_file, teardown
 
 pytestmark = pytest.mark.gpu
 
@@ -86,4 +86,4 @@ def test_random_config(ap, case):
         if writable:
             assert np.array_equal(f, cur)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)

@@ -7,7 +7,7 @@ import pytest
 import torch
 
 import oracle
-from helpers import check_invariants, make_file
+from helpers import check_invariants, make_file, teardown
 
 pytestmark = pytest.mark.gpu
 
@@ -39,7 +39,7 @@ def test_seq_writes_reach_the_file(ap, elem, frames):
         assert check_invariants(ap, cache, [r], frames) == []
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("policy,frames", [(0, 3), (1, 3), (0, 64), (1, 512)])
@@ -65,7 +65,7 @@ def test_scattered_writes_then_reads(ap, policy, frames):
         ap.ap_munmap(cache, r)  # writes back whatever is still dirty
         assert np.array_equal(f, want)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 @pytest.mark.parametrize("frames", [4, 200])
@@ -87,7 +87,7 @@ def test_apointer_copy_between_regions(ap, frames):
         ap.ap_munmap(cache, rs)
         assert np.array_equal(dst, src)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
 
 
 def test_read_only_region_rejects_writes(ap):
@@ -99,4 +99,4 @@ def test_read_only_region_rejects_writes(ap):
             ap.ap_bench_write(cache, r, ap.bench_cfg(ap.AP_SEQ, 4, 1, 32, unit_bytes=4096))
         ap.ap_munmap(cache, r)
     finally:
-        ap.ap_cache_destroy(cache)
+        teardown(ap, cache)
