@@ -529,9 +529,33 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
                                              uint64_t hint_page = 0) {
     const unsigned lane = lane_id();
     const int first = __ffs(m) - 1;
-    const unsigned wantm = __ballot_sync(m, want);
     bool got = false;
-    {
+    unsigned long long evicted = 0;
+    if (c->policy == POLICY_SEQUENTIAL && want && hint && hint_r) {
+        /* drop-behind, tried first: the frame of the page this lane's group
+         * just left (hint = frame + 1), if no pointer re-linked it meanwhile.
+         * Its entry is known (no owner-table lookup): CAS against the
+         * expected value (VALID, this frame, referenced, count 0), then once
+         * against what it holds. */
+        const uint32_t f = hint - 1;
+        uint64_t* q = AP_PTE_FIND(hint_r, hint_page);
+        if (f < c->frames && q) {
+            const uint64_t want_e = PTE_VALID | PTE_REF | ((uint64_t)f << 32);
+            const uint64_t e = pte_cas_acquire(hint_r->shared, q, want_e, PTE_EMPTY);
+            if (e == want_e) {
+                got = true;
+            } else if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f &&
+                       (e & PTE_RC_MASK) == 0 && !(e & PTE_DIRTY)) {
+                got = pte_cas_acquire(hint_r->shared, q, e, PTE_EMPTY) == e;
+            }
+            if (got) {
+                frame = f;
+                ++evicted;
+            }
+        }
+    }
+    const unsigned wantm = __ballot_sync(m, want && !got);
+    if (wantm) {
         const int k = __popc(wantm);
         const int rank = __popc(wantm & lanemask_lt());
         unsigned long long base = ~0ull;
@@ -540,39 +564,12 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
                 base = fetch_add_relaxed(c->free_head, (unsigned long long)k);
         }
         base = __shfl_sync(m, base, first);
-        if (want && base != ~0ull && base + rank < c->nfree) {
+        if (want && !got && base != ~0ull && base + rank < c->nfree) {
             frame = c->free_ids[base + rank];
             got = true;
         }
     }
     unsigned still = __ballot_sync(m, want && !got);
-    unsigned long long evicted = 0;
-    if (still && c->policy == POLICY_SEQUENTIAL) {
-        /* drop-behind: the frame of the page this lane's group just left
-         * (hint = frame + 1), if no pointer re-linked it meanwhile */
-        if (want && !got && hint && hint_r) {
-            /* the left page's entry is known (no owner-table lookup): try
-             * the CAS against its expected value (VALID, this frame,
-             * referenced, count 0), then once against what it holds */
-            const uint32_t f = hint - 1;
-            uint64_t* q = AP_PTE_FIND(hint_r, hint_page);
-            if (f < c->frames && q) {
-                const uint64_t want_e = PTE_VALID | PTE_REF | ((uint64_t)f << 32);
-                uint64_t e = pte_cas_acquire(hint_r->shared, q, want_e, PTE_EMPTY);
-                if (e == want_e) {
-                    got = true;
-                } else if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f &&
-                           (e & PTE_RC_MASK) == 0 && !(e & PTE_DIRTY)) {
-                    got = pte_cas_acquire(hint_r->shared, q, e, PTE_EMPTY) == e;
-                }
-                if (got) {
-                    frame = f;
-                    ++evicted;
-                }
-            }
-        }
-        still = __ballot_sync(m, want && !got);
-    }
     /* the lanes present (possibly fewer than 32) each examine one frame per
      * clock step; at most two laps per attempt (second chance), then back off */
     const unsigned nl = __popc(m);
@@ -744,20 +741,23 @@ struct slow_out {
  * Returns each lane's new translation and linked page; `val` receives the
  * value at the lane's offset for lanes that were unlinked. */
 /* hint (optional, per lane): bit 31 = the inline link just found this
- * lane's page EMPTY (the first round claims it without probing again); bits
- * 30:0 = frame + 1 of the page the lane's pointer left just before (hint_page
- * of the same region), for the drop-behind policy. */
+ * lane's page EMPTY (the first round claims it without probing again); bit
+ * 30 = the caller discards the value (a relink before its own loads: no
+ * value load on the way out); bits 29:0 = frame + 1 of the page the lane's
+ * pointer left just before (hint_page of the same region), for the
+ * drop-behind policy. */
 template <class T>
 __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t page,
                                                const dev_region* r, uint32_t hint = 0,
                                                uint64_t hint_page = 0) {
     bool absent = (hint >> 31) != 0;
-    hint &= 0x7fffffffu;
+    const bool want_val = ((hint >> 30) & 1u) == 0; /* bit 30: the caller discards the value */
+    hint &= 0x3fffffffu;
     /* Lanes linked on entry reload their value here, so the caller's
      * speculative load is dead on this path and is never kept live across
      * the call (keeping it live made every hit-path load wait for its data
      * before the vote's branch). */
-    T vv = (x >> 63) ? ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR)) : T{};
+    T vv = (want_val && (x >> 63)) ? ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR)) : T{};
     const dev_cache* c = r->cache;
     const unsigned lane = lane_id();
     const uint32_t lg = c->log2_page;
@@ -890,7 +890,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             page = pg;
             need = false;
             linked_here = true;
-            vv = ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
+            if (want_val) vv = ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
             progressed = true;
         }
         if ((int)lane == __ffs(m) - 1) {
@@ -1588,8 +1588,9 @@ struct ptr {
         const uint32_t hint = drop_stale(m);
         uint32_t absent = 0;
         if (__any_sync(m, !holds()) && !detail::try_link_minor<T>(m, x, page, r, lg, &absent)) {
+            /* bit 30: the caller reads the page itself (no value needed) */
             const detail::slow_out<T> o =
-                detail::deref_slow<T>(m, x, page, r, hint | (absent << 31), left);
+                detail::deref_slow<T>(m, x, page, r, hint | (absent << 31) | (1u << 30), left);
             x = o.x;
             page = o.page;
         }
