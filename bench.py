@@ -462,7 +462,7 @@ def emit_c2(args, res_all, rank, world):
                            "headline); range = pin_range (one check per page); deref = `v = *q; "
                            "q += 32` one access at a time (the paper's loop, each access checked "
                            "and able to fault; the loop issues access j+D before it uses access "
-                           "j, D = AP_DEREF_PIPE = 6, 148 CTAs of 512), overhead_vs_raw is "
+                           "j, D = AP_DEREF_PIPE = 8, 148 CTAs of 512), overhead_vs_raw is "
                            "against the tiled raw "
                            "twin, deref_vs_raw_per_access_twin against the identical per-access "
                            "loop on a raw pointer at the same launch",

@@ -160,7 +160,7 @@ __device__ __forceinline__ void seq_unit(R& q, const BenchArgs& a, uint64_t e0, 
  * the out-of-line fault path of the access that issues it (deref_slow reloads
  * lanes that were linked).  D = 1 is the plain loop. */
 #ifndef AP_DEREF_PIPE
-#define AP_DEREF_PIPE 6
+#define AP_DEREF_PIPE 8
 #endif
 template <class T, bool COPY, class R>
 __device__ __forceinline__ void seq_unit_deref(R& q, const BenchArgs& a, uint64_t e0,
@@ -203,7 +203,7 @@ __device__ __forceinline__ void seq_unit_deref(R& q, const BenchArgs& a, uint64_
 
 /* The per-access form keeps AP_DEREF_PIPE values per lane in registers
  * across the (ABI-called) fault path; built for AP_DEREF_MINB CTAs of 512
- * threads per SM (1 = 128 registers: 16 warps x 6 dereferences in flight
+ * threads per SM (1 = 128 registers: 16 warps x 8 dereferences in flight
  * measured best; 2 = 64 registers, the paper's budget, fits a
  * ring of 4).  The raw twin runs the identical loop on a plain pointer at the
  * same launch. */

@@ -31,6 +31,10 @@ for rr in raw[2:]:
               "smsp__inst_executed.sum", "lts__t_sectors_op_atom.sum", "lts__t_sectors_op_red.sum"):
         if k in d:
             print(f"raw {k} = {d[k]} {dict(zip(raw[0], raw[1])).get(k, '')}")
+    # local-memory (spill) traffic, whatever this ncu version calls it
+    for k in sorted(d):
+        if "local" in k and k.endswith(".sum") and ("inst" in k or "bytes" in k or "sectors" in k):
+            print(f"raw {k} = {d[k]} {dict(zip(raw[0], raw[1])).get(k, '')}")
     st = sorted(((float(v.replace(",", "")), k) for k, v in d.items()
                  if k.startswith("smsp__pcsamp_warps_issue_stalled") and not k.endswith("not_issued")
                  and v.replace(",", "").replace(".", "").isdigit()), reverse=True)[:8]
