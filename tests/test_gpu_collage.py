@@ -49,7 +49,8 @@ def test_index_matches_oracle(ap, K, bb):
         teardown(ap, cache)
 
 
-@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1), (1, 2), (8, 2), (1, 3), (8, 3)])
+@pytest.mark.parametrize("group,schedule", [(1, 0), (1, 1), (2, 1), (4, 0), (4, 1), (8, 0), (8, 1), (1, 2), (8, 2), (1, 3), (8, 3),
+                                            (16, 2), (32, 2), (32, 0)])
 @pytest.mark.parametrize("frames", [48, 5000])
 def test_collage_matches_oracle(ap, group, schedule, frames):
     dev = torch.device("cuda:0")
@@ -165,7 +166,8 @@ def test_collage_unit_slices_min_reduce_to_whole(ap, world, schedule):
         teardown(ap, cache)
 
 
-@pytest.mark.parametrize("group,schedule", [(1, 1), (2, 1), (4, 1), (8, 1), (4, 2), (8, 2), (8, 3)])
+@pytest.mark.parametrize("group,schedule", [(1, 1), (2, 1), (4, 1), (8, 1), (4, 2), (8, 2), (8, 3), (16, 2),
+                                            (32, 2)])
 @pytest.mark.parametrize("frames", [40, 3000])
 def test_unaligned_records_collage(ap, group, schedule, frames):
     """NEXT N1: 3 KiB histograms without padding, so records
