@@ -22,7 +22,8 @@ def read_config(name, reads):
         return dict(name="c1", file_bytes=16 << 20, page=4096, frames=64, grid=148, block=32,
                     pattern="seq", elem=16, unit=4096,
                     workload="C1: 16 MiB file, 4 KiB pages, 64-frame cache, 1 warp/SM "
-                             "sequential 16-B apointer reads, full copy out, cold per step")
+                             "sequential 16-B apointer reads (page units from a work queue), "
+                             "full copy out, cold per step")
     return dict(name="c3", file_bytes=16 * GiB, page=4096, frames=65536, grid=148, block=512,
                 pattern="divergent", elem=4, reads=max(reads // 2, 1),
                 workload="C3: divergent-warp stress, 32 lanes on 32 distinct 4 KiB pages, 256 MiB "
@@ -39,11 +40,17 @@ def run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler, host_lin
     cache = ap.ap_cache_create(cfg["frames"], cfg["page"], torch.cuda.current_device())
     region = ap.ap_mmap(cache, f)
     nthreads = cfg["grid"] * cfg["block"]
+    rr = None
     if cfg["pattern"] == "seq":
         out = torch.empty(cfg["file_bytes"], dtype=torch.uint8, device=dev)
-        bc = ap.bench_cfg(ap.AP_SEQ, cfg["elem"], cfg["grid"], cfg["block"],
+        # units from a work queue (AP_SEQ_QUEUE): with 148 warps over 64
+        # frames, round robin (AP_SEQ, measured beside it) leaves the last
+        # warps streaming alone while most frames sit idle
+        bc = ap.bench_cfg(ap.AP_SEQ_QUEUE, cfg["elem"], cfg["grid"], cfg["block"],
                           unit_bytes=cfg["unit"], out_copy=True)
-        raw = ap.bench_cfg(ap.AP_SEQ, cfg["elem"], cfg["grid"], cfg["block"],
+        rr = ap.bench_cfg(ap.AP_SEQ, cfg["elem"], cfg["grid"], cfg["block"],
+                          unit_bytes=cfg["unit"], out_copy=True)
+        raw = ap.bench_cfg(ap.AP_SEQ_QUEUE, cfg["elem"], cfg["grid"], cfg["block"],
                            unit_bytes=cfg["unit"], out_copy=True, mode=ap.AP_MODE_RAW,
                            raw_base=ap.ap_region_devptr(cache, region))
         reads = cfg["file_bytes"] // cfg["elem"]
@@ -92,6 +99,17 @@ def run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler, host_lin
         other[name] = dict(s=min(to), fill_GBps=so["fill_bytes"] / min(to) / 1e9,
                            evictions=so["evictions"], equal=bool(torch.equal(out_o, out)))
         ap.ap_cache_set_policy(cache, pol_names[policy])
+    if rr is not None:
+        out_o = torch.empty_like(out)
+        to = []
+        for _ in range(3):
+            ap.ap_cache_reset(cache)
+            to.append(timed(torch, lambda: ap.ap_bench_read(cache, region, rr, out_o, stream),
+                            stream))
+        so = ap.ap_cache_stats(cache)
+        other["round_robin_units"] = dict(s=min(to), fill_GBps=so["fill_bytes"] / min(to) / 1e9,
+                                          evictions=so["evictions"],
+                                          equal=bool(torch.equal(out_o, out)))
     out_raw = torch.empty_like(out)
     raw_t = min(timed(torch, lambda: ap.ap_bench_read(cache, region, raw, out_raw, stream), stream)
                 for _ in range(3))

@@ -215,13 +215,16 @@ int ap_prefill(ap_cache_t cache, ap_region_t region, uint64_t first_page, uint64
 #define AP_SEQ 0       /* warp w reads units w, w+W, ... sequentially         */
 #define AP_UNIFORM 1   /* uniform-random element offsets                      */
 #define AP_DIVERGENT 2 /* the 32 lanes of a warp on 32 distinct pages         */
+#define AP_SEQ_QUEUE 3 /* AP_SEQ's units, handed out in order from a device   *
+                        * counter (the next free warp takes the next unit);    *
+                        * out_copy and AP_ACCESS_TILE only                     */
 
 #define AP_MODE_APOINTER 0 /* read through ap::ptr<T> (the method)           */
 #define AP_MODE_RAW 1      /* identical kernel on a raw pointer (the twin,     *
                             * PAPER.md:304 "two versions of every benchmark") */
 
 typedef struct {
-    int32_t pattern;           /* AP_SEQ | AP_UNIFORM | AP_DIVERGENT             */
+    int32_t pattern;           /* AP_SEQ | AP_UNIFORM | AP_DIVERGENT | AP_SEQ_QUEUE */
     uint32_t elem_bytes;       /* 4, 8 or 16                                     */
     uint32_t grid, block;      /* launch shape; block a multiple of 32, <= 1024  */
     uint32_t reads_per_thread; /* UNIFORM / DIVERGENT                            */

@@ -197,6 +197,15 @@ struct alignas(64) dev_cache {
     uint32_t backoff_min_ns; /* fault-path back-off: exponential from min to max */
     uint32_t backoff_max_ns;
 };
+/* dev_region::prot bit: the cache runs AP_POLICY_SEQUENTIAL, so a warp that
+ * leaves a page with all its lanes keeps one reference on it (the
+ * drop-behind pin) until its fault path has taken the frame over or let it
+ * go (ptr::drop_stale, deref_slow) */
+constexpr uint32_t REGION_DROP_BEHIND = 1u << 8;
+/* deref_slow hint bits: the warp pins the page it left with one reference;
+ * the lane (a group leader) already claimed its page (LOADING) inline */
+constexpr uint32_t HINT_PINNED = 1u << 29;
+constexpr uint32_t HINT_CLAIMED = 1u << 28;
 
 /* ---------------------------------------------------- PTX helpers (A15) */
 namespace detail {
@@ -221,6 +230,20 @@ __device__ __forceinline__ uint64_t now_ns() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+/* AP_FAULT_PROF (diagnostic builds only, tools/exp_fault_phases.py): SM
+ * cycles per fault-path phase, summed by each warp's first lane into
+ * ap_fprof (defined in ap_runtime.cu, read by ap_fault_prof). */
+#ifdef AP_FAULT_PROF
+extern __device__ unsigned long long ap_fprof[16];
+#define AP_FP_T(v) const long long v = clock64()
+#define AP_FP_ADD(m, i, d)                                                              \
+    do {                                                                                \
+        if (::ap::detail::lane_id() == (unsigned)(__ffs(m) - 1)) atomicAdd(&::ap::detail::ap_fprof[i], (unsigned long long)(d)); \
+    } while (0)
+#else
+#define AP_FP_T(v)
+#define AP_FP_ADD(m, i, d)
+#endif
 __device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
     uint64_t v;
     asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -484,6 +507,34 @@ static __device__ AP_UNLINK_ATTR void unlink_lanes(unsigned m, bool mine, const 
     AP_PT_RECONVERGE(m);
 }
 
+/* Drop-behind unlink (AP_POLICY_SEQUENTIAL, R-A11b): when every lane of m
+ * leaves the same page, the warp keeps one of its n references (the pin:
+ * no other warp can evict the page, so no sweep takes the frame between
+ * this unlink and the warp's own fault) and drops n - 1 with a relaxed add
+ * (the pin keeps the frame, so no release is needed).  The fault path then
+ * takes the frame over with one CAS (count 1 -> EMPTY) or drops the pin.
+ * Returns true (for every lane) if the warp pinned the page; otherwise it
+ * is unlink_lanes. */
+static __device__ __forceinline__ bool unlink_lanes_pin(unsigned m, bool mine, const dev_region* r,
+                                                        uint64_t page) {
+#ifdef AP_PT_HASH
+    unlink_lanes(m, mine, r, page);
+    return false;
+#else
+    unsigned long long key = mine ? (((unsigned long long)r->id << 48) | page) : ~0ull;
+    const unsigned grp = __match_any_sync(m, key);
+    const bool keep = mine && grp == m && !r->shared;
+    if (mine && lane_id() == (unsigned)(__ffs(grp) - 1)) {
+        const unsigned n = __popc(grp);
+        if (!keep) red_unlink(AP_PTE_AT(r, page), (uint64_t)0 - (uint64_t)n);
+        else if (n > 1)
+            red_add_relaxed(reinterpret_cast<unsigned long long*>(AP_PTE_AT(r, page)),
+                            (unsigned long long)(0 - (uint64_t)(n - 1)));
+    }
+    return keep;
+#endif
+}
+
 /* -------------------------------------------------------------------------
  * Write-back (writable mappings, NEXT N3): the lanes in m copy frame f to
  * the page's bytes in host memory over the host link (zero-copy 16-B
@@ -523,34 +574,53 @@ __device__ __forceinline__ void writeback_page(unsigned m, const dev_cache* c, c
  * 113, 145); the clock gives referenced pages a second chance (R-A11).  A
  * victim is claimed by CAS of its PTE (VALID, rc=0) -> EMPTY, which a
  * concurrent minor fault's CAS either precedes or loses to. */
+/* descriptor fields the fault path loads once on entry (see deref_slow) */
+struct fault_hot {
+    int32_t policy;
+    uint64_t frames;
+    dev_stats* stats;
+    uint64_t* pte;   /* hint_r's page table (dense build) */
+    uint32_t shared; /* hint_r->shared */
+};
 __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, bool want,
                                              uint32_t& frame, uint32_t hint = 0,
                                              const dev_region* hint_r = nullptr,
-                                             uint64_t hint_page = 0) {
+                                             uint64_t hint_page = 0, uint64_t pin = 0,
+                                             bool* took_hint = nullptr,
+                                             const fault_hot* hot = nullptr) {
     const unsigned lane = lane_id();
     const int first = __ffs(m) - 1;
     bool got = false;
     unsigned long long evicted = 0;
-    if (c->policy == POLICY_SEQUENTIAL && want && hint && hint_r) {
+    const int32_t policy = hot ? hot->policy : c->policy;
+    const uint64_t nframes = hot ? hot->frames : c->frames;
+    if (policy == POLICY_SEQUENTIAL && want && hint && hint_r) {
         /* drop-behind, tried first: the frame of the page this lane's group
          * just left (hint = frame + 1), if no pointer re-linked it meanwhile.
          * Its entry is known (no owner-table lookup): CAS against the
-         * expected value (VALID, this frame, referenced, count 0), then once
-         * against what it holds. */
+         * expected value (VALID, this frame, referenced, count = the warp's
+         * drop-behind pin (1) or 0), then once against what it holds. */
         const uint32_t f = hint - 1;
+#ifdef AP_PT_HASH
         uint64_t* q = AP_PTE_FIND(hint_r, hint_page);
-        if (f < c->frames && q) {
-            const uint64_t want_e = PTE_VALID | PTE_REF | ((uint64_t)f << 32);
-            const uint64_t e = pte_cas_acquire(hint_r->shared, q, want_e, PTE_EMPTY);
+        const uint32_t hshared = hint_r->shared;
+#else
+        uint64_t* q = hot ? hot->pte + hint_page : AP_PTE_FIND(hint_r, hint_page);
+        const uint32_t hshared = hot ? hot->shared : hint_r->shared;
+#endif
+        if (f < nframes && q) {
+            const uint64_t want_e = PTE_VALID | PTE_REF | ((uint64_t)f << 32) | pin;
+            uint64_t e = pte_cas_acquire(hshared, q, want_e, PTE_EMPTY);
             if (e == want_e) {
                 got = true;
             } else if ((e >> 62) == 2 && ((e >> 32) & PTE_FRAME_MASK) == f &&
-                       (e & PTE_RC_MASK) == 0 && !(e & PTE_DIRTY)) {
-                got = pte_cas_acquire(hint_r->shared, q, e, PTE_EMPTY) == e;
+                       (e & PTE_RC_MASK) == pin && !(e & PTE_DIRTY)) {
+                got = pte_cas_acquire(hshared, q, e, PTE_EMPTY) == e;
             }
             if (got) {
                 frame = f;
                 ++evicted;
+                if (took_hint) *took_hint = true;
             }
         }
     }
@@ -635,8 +705,9 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
         still = __ballot_sync(m, want && !got);
     }
     if ((int)lane == first) {
-        stat_add(&my_stats(c)->evictions, evicted);
-        if (still) stat_add(&my_stats(c)->nofree, 1);
+        dev_stats* S = hot ? hot->stats : my_stats(c);
+        stat_add(&S->evictions, evicted);
+        if (still) stat_add(&S->nofree, 1);
     }
 #ifdef AP_DEBUG
     if (still && (int)lane == first) {
@@ -657,13 +728,13 @@ __device__ __forceinline__ bool alloc_frames(const dev_cache* c, unsigned m, boo
  * from pinned host memory over the host link (zero copy) or, for N2, from a
  * peer cache's frame; the first `len` bytes come from `src` and a ragged
  * last page is zero-padded.  Host bytes are 16-B aligned (ap_mmap checks it). */
-__device__ __forceinline__ void fill_page(unsigned m, const dev_cache* c, uint64_t f,
+__device__ __forceinline__ void fill_page(unsigned m, uint8_t* pool, uint32_t lg, uint64_t f,
                                           const uint8_t* src, uint64_t len) {
     /* the lanes in m share the copy: rank = position among them */
     const unsigned lane = __popc(m & lanemask_lt());
     const unsigned nl = __popc(m);
-    const uint64_t P = 1ull << c->log2_page;
-    uint8_t* dst = c->pool + f * P;
+    const uint64_t P = 1ull << lg;
+    uint8_t* dst = pool + f * P;
     const uint64_t nvec = len / 16;
     const uint4* s4 = reinterpret_cast<const uint4*>(src);
     uint4* d4 = reinterpret_cast<uint4*>(dst);
@@ -752,7 +823,12 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
                                                uint64_t hint_page = 0) {
     bool absent = (hint >> 31) != 0;
     const bool want_val = ((hint >> 30) & 1u) == 0; /* bit 30: the caller discards the value */
-    hint &= 0x3fffffffu;
+    /* HINT_PINNED: the warp still holds one reference on hint_page (the
+     * drop-behind pin, ptr::drop_stale); round 1 hands it to the frame
+     * allocation or drops it before anything can wait */
+    bool pinned = (hint & HINT_PINNED) != 0;
+    bool claimed_in = (hint & HINT_CLAIMED) != 0;
+    hint &= 0x0fffffffu;
     /* Lanes linked on entry reload their value here, so the caller's
      * speculative load is dead on this path and is never kept live across
      * the call (keeping it live made every hit-path load wait for its data
@@ -762,24 +838,47 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
     const unsigned lane = lane_id();
     const uint32_t lg = c->log2_page;
     const uint64_t P = 1ull << lg;
+    dev_stats* S = my_stats(c);
+    /* descriptor fields the rounds use, loaded once here: each acquire below
+     * invalidates L1, so a field first read after one would cost an L2
+     * round trip on the fault's critical path */
+#ifdef AP_PT_HASH
+    const fault_hot hot{c->policy, c->frames, S, nullptr, r->shared};
+#else
+    const fault_hot hot{c->policy, c->frames, S, r->pte, r->shared};
+#endif
+    const uint32_t max_claims = c->max_claims;
+    uint64_t* const owner_tab = c->owner;
+    uint8_t* const pool = c->pool;
+    const uint8_t* const r_host = r->host;
+    const uint64_t r_bytes = r->bytes;
+    const uint32_t r_npeers = r->npeers;
+    const uint32_t r_shared = r->shared;
+    const uint32_t r_id = r->id;
+#ifndef AP_PT_HASH
+    uint64_t* const r_pte = r->pte;
+#endif
     bool need = !(x >> 63);
-    if (need && (x + sizeof(T) > r->bytes || (x % sizeof(T)) != 0)) {
+    if (need && (x + sizeof(T) > r_bytes || (x % sizeof(T)) != 0)) {
         set_err(c, ERR_FAULT);
         vv = T{};
         need = false;
     }
     const uint64_t pg = need ? (x >> lg) : 0;
-    const unsigned long long mykey = ((unsigned long long)r->id << 48) | pg;
+    const unsigned long long mykey = ((unsigned long long)r_id << 48) | pg;
     bool linked_here = false;
     bool held = !need && (x >> 63); /* linked before this call: value already loaded */
     uint64_t t0 = 0;
     uint32_t backoff = c->backoff_min_ns;
     int idle_rounds = 0;
-    dev_stats* S = my_stats(c);
+    AP_FP_T(tp_entry);
+    AP_FP_ADD(m, 0, 1);
 
     for (;;) {
         const unsigned pend = __ballot_sync(m, need);
         if (!pend) break;
+        AP_FP_T(tp0);
+        AP_FP_ADD(m, 7, 1);
         const unsigned grp = __match_any_sync(m, need ? mykey : ~0ull);
         const int leader = __ffs(grp) - 1;
         const bool is_leader = need && (int)lane == leader;
@@ -788,7 +887,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         uint64_t* pte = is_leader ? pt_find(r, pg, true) : nullptr;
         __syncwarp(m);
 #else
-        uint64_t* pte = r->pte + pg;
+        uint64_t* pte = r_pte + pg;
 #endif
 
         /* Phase A (leaders, lane-parallel; R-A13): minor faults link at once;
@@ -804,7 +903,9 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         /* first round after an inline link found the page EMPTY: go straight
          * to the claim (a race with a concurrent claim or publish just makes
          * the CAS fail and the next round probe again) */
-        const bool probed = is_leader && !absent;
+        const bool pre_claimed = is_leader && claimed_in; /* link_minor claimed it */
+        claimed_in = false;
+        const bool probed = is_leader && !absent && !pre_claimed;
         uint64_t old = probed ? add_link(pte, n) : 0;
         absent = false;
 #ifdef AP_DEBUG
@@ -822,13 +923,15 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         }
         const unsigned empties = __ballot_sync(m, is_leader && (old >> 62) == 0);
         const bool may_claim = !((empties >> lane) & 1u) ||
-                               (uint32_t)__popc(empties & lanemask_lt()) < c->max_claims;
-        if (is_leader && st == ST_NONE) {
+                               (uint32_t)__popc(empties & lanemask_lt()) < max_claims;
+        if (pre_claimed) {
+            st = ST_CLAIMED;
+        } else if (is_leader && st == ST_NONE) {
             if ((old >> 62) == 0) {
                 if (!may_claim) {
                     st = ST_SKIP;
                 } else {
-                    const uint64_t prev = pte_cas_acquire(r->shared, pte, PTE_EMPTY, PTE_LOADING);
+                    const uint64_t prev = pte_cas_acquire(r_shared, pte, PTE_EMPTY, PTE_LOADING);
                     /* prev != 0: transient counts, a racing claimer or a
                      * publish in between; all resolve by retrying */
                     st = prev == PTE_EMPTY ? ST_CLAIMED : ST_WAIT;
@@ -840,13 +943,24 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
 
         /* Phase B: frames for the claimed pages (S7). */
         const unsigned claimed = __ballot_sync(m, st == ST_CLAIMED);
+        AP_FP_T(tp1);
+        AP_FP_ADD(m, 1, tp1 - tp0);
+        bool took_pin = false;
         if (claimed) {
-            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame, hint, r, hint_page);
+            const bool ok = alloc_frames(c, m, st == ST_CLAIMED, frame, hint, r, hint_page,
+                                         pinned ? 1 : 0, &took_pin, &hot);
             if (st == ST_CLAIMED && !ok) {
                 /* give the page back (an add, so transient counts survive) */
-                pte_red_release(r->shared, pte, (uint64_t)0 - PTE_LOADING);
+                pte_red_release(r_shared, pte, (uint64_t)0 - PTE_LOADING);
                 st = ST_NOFRAME;
             }
+        }
+        if (pinned) {
+            /* the pin was not taken over with its frame: drop it (release:
+             * the warp's reads of that page are done) */
+            if (!__any_sync(m, took_pin) && (int)lane == __ffs(m) - 1)
+                red_unlink(AP_PTE_AT(r, hint_page), (uint64_t)0 - 1);
+            pinned = false;
         }
 
         /* Phase C: fills, one page at a time by the whole warp (S8), then the
@@ -854,31 +968,45 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
          * leader release-stores VALID with the group's count. */
         unsigned fill = __ballot_sync(m, st == ST_CLAIMED);
         const int nfill = __popc(fill);
+        AP_FP_T(tp2);
+        AP_FP_ADD(m, 2, tp2 - tp1);
         while (fill) {
             const int L = __ffs(fill) - 1;
             fill &= fill - 1;
             const uint32_t f = __shfl_sync(m, frame, L);
             const uint64_t fpg = __shfl_sync(m, pg, L);
-            const dev_region* fr =
-                reinterpret_cast<const dev_region*>(__shfl_sync(m, (unsigned long long)r, L));
-            if ((int)lane == L) st_relaxed(c->owner + f, ((uint64_t)(fr->id + 1) << 48) | fpg);
-                        const uint8_t* src = fr->host + (fpg << lg);
-            const uint64_t avail = fr->bytes - (fpg << lg);
-            uint64_t* peer_q = fr->npeers ? peer_pin(m, c, fr, fpg, &src) : nullptr;
-            fill_page(m, c, f, src, peer_q ? P : (avail < P ? avail : P));
+            /* the filling lane's region (lanes may point into different
+             * regions): its fields from that lane's registers */
+            const uint32_t fid = __shfl_sync(m, r_id, L);
+            const uint8_t* src = reinterpret_cast<const uint8_t*>(
+                                     __shfl_sync(m, (unsigned long long)r_host, L)) + (fpg << lg);
+            const uint64_t avail = __shfl_sync(m, (unsigned long long)r_bytes, L) - (fpg << lg);
+            if ((int)lane == L) st_relaxed(owner_tab + f, ((uint64_t)(fid + 1) << 48) | fpg);
+            uint64_t* peer_q = nullptr;
+            if (__shfl_sync(m, r_npeers, L)) {
+                const dev_region* fr =
+                    reinterpret_cast<const dev_region*>(__shfl_sync(m, (unsigned long long)r, L));
+                peer_q = peer_pin(m, c, fr, fpg, &src);
+            }
+            fill_page(m, pool, lg, f, src, peer_q ? P : (avail < P ? avail : P));
             if (peer_q) peer_unpin(m, c, peer_q);
             else if ((int)lane == __ffs(m) - 1) stat_add(&S->fill_bytes, avail < P ? avail : P);
+            AP_FP_T(tp3);
+            AP_FP_ADD(m, 3, tp3 - tp2);
             fence_gpu();
             __syncwarp(m);
+            AP_FP_T(tp4);
+            AP_FP_ADD(m, 4, tp4 - tp3);
 #ifdef AP_DEBUG
             if ((int)lane == L) printf("[publish] w%u m%08x n%u f%u pg %llu\n", (unsigned)(threadIdx.x >> 5), m, n, f, (unsigned long long)fpg);
 #endif
             if ((int)lane == L)
-                pte_red_release(fr->shared, pte,
+                pte_red_release(r_shared, pte,
                                 (PTE_VALID - PTE_LOADING) | (AP_REF_ON_FILL ? PTE_REF : 0) |
                                     ((uint64_t)f << 32) | (uint64_t)n);
         }
         const unsigned nminor = __popc(__ballot_sync(m, st == ST_LINKED));
+        AP_FP_T(tp5);
 
         /* Phase D: link the group lanes and read their values (S9). */
         const int lst = __shfl_sync(m, st, leader);
@@ -886,7 +1014,7 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
         __syncwarp(m);
         bool progressed = false;
         if (need && (lst == ST_LINKED || lst == ST_CLAIMED)) {
-            x = XL_VALID | ((uint64_t)(c->pool + (uint64_t)lf * P) + (x & (P - 1)));
+            x = XL_VALID | ((uint64_t)(pool + (uint64_t)lf * P) + (x & (P - 1)));
             page = pg;
             need = false;
             linked_here = true;
@@ -898,6 +1026,8 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             stat_add(&S->minor, nminor);
         }
         progressed = __any_sync(m, progressed);
+        AP_FP_T(tp6);
+        AP_FP_ADD(m, 5, tp6 - tp5);
 
         /* Lanes still unserved: either skipped (another claim this round),
          * waiting on a page another warp is loading, or out of frames. */
@@ -946,6 +1076,10 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
             }
         }
     }
+    if (pinned && (int)lane == __ffs(m) - 1) /* no round ran (every lane out of range) */
+        red_unlink(AP_PTE_AT(r, hint_page), (uint64_t)0 - 1);
+    AP_FP_T(tp_exit);
+    AP_FP_ADD(m, 6, tp_exit - tp_entry);
     return slow_out<T>{x, page, vv};
 }
 
@@ -971,13 +1105,22 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
     const int leader = __ffs(grp) - 1;
     const bool is_leader = need && (int)lane_id() == leader;
     uint64_t old = 0;
+    bool claimed = false;
     if (is_leader) {
 #ifdef AP_PT_HASH
         uint64_t* pte = pt_find(r, pg, false); /* no slot: not resident */
         if (pte) {
 #else
         uint64_t* pte = r->pte + pg;
-        {
+        /* a sequential stream (drop-behind policy) expects its next page to
+         * be absent: probe with the claim (EMPTY -> LOADING, the fault
+         * path's first step) and link with the add only if it is VALID */
+        const bool stream = (r->prot & REGION_DROP_BEHIND) && !r->shared;
+        if (stream) {
+            old = cas_acquire(pte, PTE_EMPTY, PTE_LOADING);
+            claimed = old == PTE_EMPTY;
+        }
+        if (!claimed && (!stream || (old >> 62) == 2)) {
 #endif
             old = add_link(pte, __popc(grp));
             if ((old >> 62) == 2) {
@@ -1002,9 +1145,15 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
         x = XL_VALID | ((uint64_t)(r->pool + f * P) + (x & (P - 1)));
         page = pg;
     }
-    /* the page was not resident (EMPTY): the fault path may claim it at once */
-    if (absent) *absent = (need && (old >> 62) == 0) ? 1u : 0u;
+    /* the page was not resident (EMPTY): the fault path may claim it at once
+     * (bit 0); this lane, its group's leader, claimed it already (bit 1) */
+    if (absent) *absent = (need && (old >> 62) == 0 ? 1u : 0u) | (claimed ? 2u : 0u);
     return __all_sync(m, ok);
+}
+
+/* link_minor's `absent` bits as deref_slow hint bits */
+__device__ __forceinline__ uint32_t absent_hint(uint32_t absent) {
+    return ((absent & 1u) << 31) | ((absent & 2u) ? HINT_CLAIMED : 0u);
 }
 
 /* link_minor unless built with -DAP_NO_LINK_MINOR (ablation: every link
@@ -1287,14 +1436,15 @@ struct ptr {
      * resident (link_minor), else through the fault handler. */
     __device__ __forceinline__ T deref_miss(unsigned m) {
         const uint64_t left = page;
-        const uint32_t hint = drop_stale(m);
+        const uint32_t hint = drop_stale(m, true);
         uint32_t absent = 0;
         if (detail::try_link_minor<T>(m, x, page, r, lg, &absent)) {
             sync_fb();
+            unpin(m, hint, left);
             return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
         }
         const detail::slow_out<T> o =
-            detail::deref_slow<T>(m, x, page, r, hint | (absent << 31), left);
+            detail::deref_slow<T>(m, x, page, r, hint | detail::absent_hint(absent), left);
         x = o.x;
         page = o.page;
         sync_fb();
@@ -1568,13 +1718,26 @@ struct ptr {
     }
     /* lanes that walked off their frame unlink it and carry
      * on unlinked at the same file offset */
-    __device__ __forceinline__ uint32_t drop_stale(unsigned m) {
+    /* drop the drop-behind pin on page `left` when no fault follows */
+    __device__ __forceinline__ void unpin(unsigned m, uint32_t hint, uint64_t left) {
+        if ((hint & HINT_PINNED) && detail::lane_id() == (unsigned)(__ffs(m) - 1))
+            detail::red_unlink(AP_PTE_AT(r, left), (uint64_t)0 - 1);
+    }
+    /* pin: the caller is a read fault path that passes the hint on to
+     * deref_slow (or drops the pin itself): under drop-behind a warp that
+     * leaves one page with all its lanes keeps one reference on it
+     * (HINT_PINNED) */
+    __device__ __forceinline__ uint32_t drop_stale(unsigned m, bool pin = false) {
         const bool stale = holds() && !ready();
         uint32_t hint = 0; /* the dropped frame + 1 (drop-behind policy) */
         if (__any_sync(m, stale)) {
             const uint64_t off = foff();
             if (stale) hint = (uint32_t)((((fb & XL_ADDR) - (uint64_t)r->pool) >> lg) + 1);
-            detail::unlink_lanes(m, stale, r, page);
+            if (pin && (r->prot & REGION_DROP_BEHIND)) {
+                if (detail::unlink_lanes_pin(m, stale, r, page)) hint |= HINT_PINNED;
+            } else {
+                detail::unlink_lanes(m, stale, r, page);
+            }
             if (stale) {
                 x = off;
                 fb = XL_VALID;
@@ -1585,12 +1748,20 @@ struct ptr {
     /* make every lane of m linked at its current offset */
     __device__ __forceinline__ void relink(unsigned m) {
         const uint64_t left = page;
-        const uint32_t hint = drop_stale(m);
+        AP_FP_T(tr0);
+        const uint32_t hint = drop_stale(m, true);
+        AP_FP_T(tr1);
+        AP_FP_ADD(m, 8, tr1 - tr0);
         uint32_t absent = 0;
-        if (__any_sync(m, !holds()) && !detail::try_link_minor<T>(m, x, page, r, lg, &absent)) {
+        const bool minor_ok = !__any_sync(m, !holds()) || detail::try_link_minor<T>(m, x, page, r, lg, &absent);
+        AP_FP_T(tr2);
+        AP_FP_ADD(m, 9, tr2 - tr1);
+        AP_FP_ADD(m, 10, 1);
+        if (minor_ok) unpin(m, hint, left);
+        if (!minor_ok) {
             /* bit 30: the caller reads the page itself (no value needed) */
             const detail::slow_out<T> o =
-                detail::deref_slow<T>(m, x, page, r, hint | (absent << 31) | (1u << 30), left);
+                detail::deref_slow<T>(m, x, page, r, hint | detail::absent_hint(absent) | (1u << 30), left);
             x = o.x;
             page = o.page;
         }

@@ -10,7 +10,7 @@ import numpy as np
 
 from . import _lib
 from ._lib import (AP_PROT_READ, AP_PROT_WRITE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_AHEAD, AP_ACCESS_PAIR, AP_ACCESS_TMA, AP_ACCESS_TILE, AP_DIVERGENT, AP_MODE_APOINTER, AP_MODE_RAW, AP_POLICY_CLOCK, AP_POLICY_SEQUENTIAL,  # noqa: F401
-                   AP_POLICY_RANDOM, AP_SCHED_LSH, AP_SCHED_NATURAL, AP_SCHED_TABLE, AP_SCHED_TABLE_MH, AP_SEQ,
+                   AP_POLICY_RANDOM, AP_SCHED_LSH, AP_SCHED_NATURAL, AP_SCHED_TABLE, AP_SCHED_TABLE_MH, AP_SEQ, AP_SEQ_QUEUE,
                    AP_UNIFORM, APError, ap_bench_cfg, ap_collage_in,
                    ap_stats_t, AP_COLLAGE_ACCUMULATE, AP_COLLAGE_SYSTEM, AP_PART_BLOCKS,
                    AP_PART_RECORDS, AP_PART_UNITS, AP_MGPU_MAX, ap_ipc_handle_t,

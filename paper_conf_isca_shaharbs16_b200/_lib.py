@@ -13,7 +13,7 @@ AP_OK = 0
 AP_EINVAL, AP_ENOMEM, AP_ECUDA, AP_EBUSY, AP_ERANGE = -1, -2, -3, -4, -5
 AP_EFAULT, AP_ENOFRAME, AP_ETIMEDOUT = -6, -7, -8
 AP_POLICY_CLOCK, AP_POLICY_RANDOM, AP_POLICY_SEQUENTIAL = 0, 1, 2
-AP_SEQ, AP_UNIFORM, AP_DIVERGENT = 0, 1, 2
+AP_SEQ, AP_UNIFORM, AP_DIVERGENT, AP_SEQ_QUEUE = 0, 1, 2, 3
 AP_MODE_APOINTER, AP_MODE_RAW = 0, 1
 AP_ACCESS_TILE, AP_ACCESS_DEREF, AP_ACCESS_RANGE, AP_ACCESS_AHEAD, AP_ACCESS_PAIR, AP_ACCESS_TMA = 0, 1, 2, 3, 4, 5
 AP_SCHED_NATURAL, AP_SCHED_LSH, AP_SCHED_TABLE, AP_SCHED_TABLE_MH = 0, 1, 2, 3

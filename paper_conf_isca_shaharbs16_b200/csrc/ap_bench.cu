@@ -61,6 +61,7 @@ struct BenchArgs {
     uint8_t* out_copy;  /* SEQ copy output or nullptr                   */
     int32_t access;     /* AP_ACCESS_*                                  */
     uint64_t* ck;       /* per-thread checksums                         */
+    unsigned long long* queue; /* AP_SEQ_QUEUE: next unit (zeroed per launch) */
 };
 
 __device__ __forceinline__ uint64_t uniform_off(const BenchArgs& a, uint32_t E, uint64_t t,
@@ -366,6 +367,44 @@ __global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
     if (!a.out_copy) a.ck[t] = h;
 }
 
+/* AP_SEQ_QUEUE: the k_seq stream with units handed out in order from a
+ * device counter instead of round robin, so warps that hold frames keep
+ * streaming while warps waiting for one hold a single unit (C1: 148 warps
+ * over 64 frames; round robin leaves the last warps to finish alone).  The
+ * next unit's index is fetched while the current one is read.  Copy output
+ * only (the bytes land at their offsets whichever warp reads them). */
+template <class T, bool APTR>
+__global__ void __launch_bounds__(AP_BENCH_THREADS, AP_SEQ_MINB)
+    k_seq_queue(const ap::dev_cache* __restrict__ c, uint32_t region, const BenchArgs a) {
+    constexpr uint32_t E = sizeof(T);
+    const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t lane = t & 31;
+    const uint64_t nunits = (a.span + a.unit - 1) / a.unit;
+    const uint64_t total = nunits * a.passes;
+    const uint32_t per_unit = a.unit / (32 * E);
+    uint64_t h = FNV_BASIS;
+    [[maybe_unused]] ap::ptr<T> q;
+    if constexpr (APTR) q = ap::gvmmap<T>(c, region, 0);
+    unsigned long long v = 0;
+    if (lane == 0) v = atomicAdd(a.queue, 1ull);
+    v = __shfl_sync(0xffffffffu, v, 0);
+    while (v < total) {
+        unsigned long long vn = 0;
+        if (lane == 0) vn = atomicAdd(a.queue, 1ull);
+        const uint64_t u = v % nunits;
+        const uint64_t e0 = u * (a.unit / E) + lane;
+        const bool whole = (u + 1) * a.unit <= a.span;
+        if constexpr (APTR) {
+            q += (int64_t)(e0 * E - q.foff()) / (int64_t)E;
+            seq_unit<T>(q, a, e0, per_unit, whole, h);
+        } else {
+            raw_reader<T> q{reinterpret_cast<const T*>(a.raw) + e0};
+            seq_unit<T>(q, a, e0, per_unit, whole, h);
+        }
+        v = __shfl_sync(0xffffffffu, vn, 0);
+    }
+}
+
 /* The split-phase link experiments (AP_ACCESS_AHEAD, AP_ACCESS_PAIR) get a
  * kernel of their own, so adding them does not perturb ptxas's allocation of
  * k_seq's tile loop (tests/test_sass.py). */
@@ -526,6 +565,12 @@ cudaError_t launch_t(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg
             else
                 k_seq<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             break;
+        case AP_SEQ_QUEUE: {
+            const cudaError_t e = cudaMemsetAsync(a.queue, 0, sizeof(unsigned long long), s);
+            if (e != cudaSuccess) return e;
+            k_seq_queue<T, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
+            break;
+        }
         case AP_UNIFORM:
             k_random<T, AP_UNIFORM, APTR><<<cfg->grid, cfg->block, 0, s>>>(c->d_cache, region, a);
             break;
@@ -575,6 +620,11 @@ int make_args(const ap_cache_s* c, ap_region_t region, const ap_bench_cfg* cfg, 
         return AP_EINVAL;
 #endif
     switch (cfg->pattern) {
+        case AP_SEQ_QUEUE:
+            /* copy output, tile access: the queue's unit order is dynamic */
+            if (!cfg->out_copy || cfg->access != AP_ACCESS_TILE) return AP_EINVAL;
+            a->queue = c->seq_queue;
+            [[fallthrough]];
         case AP_SEQ:
             if (a->unit == 0 || a->unit % (32 * E) || a->span > rg.bytes) return AP_EINVAL;
             if (cfg->mode == AP_MODE_APOINTER && (c->page % a->unit)) return AP_EINVAL;
@@ -628,7 +678,7 @@ extern "C" int ap_bench_read_host(ap_cache_t c, ap_region_t region, const ap_ben
     ap_device_guard g(c->device);
     const uint64_t nthreads = (uint64_t)cfg->grid * cfg->block;
     uint64_t out_bytes = nthreads * 8;
-    if (cfg->pattern == AP_SEQ && cfg->out_copy)
+    if ((cfg->pattern == AP_SEQ || cfg->pattern == AP_SEQ_QUEUE) && cfg->out_copy)
         out_bytes = cfg->span_bytes ? cfg->span_bytes : c->reg[region].bytes;
     void* d = nullptr;
     AP_CUDA_TRY(cudaMalloc(&d, out_bytes));

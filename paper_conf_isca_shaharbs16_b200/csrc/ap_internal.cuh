@@ -45,6 +45,7 @@ struct ap_cache_s {
     uint32_t* free_ids = nullptr;
     unsigned long long* free_head = nullptr;
     unsigned long long* clock_hand = nullptr;
+    unsigned long long* seq_queue = nullptr; /* AP_SEQ_QUEUE unit counter */
     ap::dev_region* regions = nullptr;
     ap::dev_stats* stats = nullptr;
     int* err = nullptr;

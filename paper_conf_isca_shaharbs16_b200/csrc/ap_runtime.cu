@@ -64,6 +64,12 @@ bool ap_region_ok(const ap_cache_s* c, ap_region_t r) {
     return c && r < c->reg.size() && c->reg[r].live;
 }
 
+/* the device copy of a region's prot: + REGION_DROP_BEHIND under
+ * AP_POLICY_SEQUENTIAL (read by a pointer's unlink when it leaves a page) */
+static uint32_t region_prot_flags(const ap_cache_s* c, uint32_t prot) {
+    return prot | (c->h.policy == ap::POLICY_SEQUENTIAL ? ap::REGION_DROP_BEHIND : 0u);
+}
+
 static int push_descriptor(ap_cache_s* c) {
     AP_CUDA_TRY(cudaMemcpy(c->d_cache, &c->h, sizeof(ap::dev_cache), cudaMemcpyHostToDevice));
     return AP_OK;
@@ -229,6 +235,7 @@ extern "C" int ap_cache_create(uint64_t frames, uint32_t page_size, int device, 
     if (cudaMalloc(&c->free_head, 256) != cudaSuccess) return fail(AP_ENOMEM);
     c->clock_hand = c->free_head + 8;
     c->err = (int*)(c->free_head + 16);
+    c->seq_queue = c->free_head + 24;
     if (cudaMalloc(&c->regions, sizeof(ap::dev_region) * AP_MAX_REGIONS) != cudaSuccess)
         return fail(AP_ENOMEM);
     if (cudaMalloc(&c->stats, sizeof(ap::dev_stats) * ap::STAT_SHARDS) != cudaSuccess)
@@ -472,7 +479,7 @@ extern "C" int ap_mmap_prot(ap_cache_t c, const void* host_buf, uint64_t bytes, 
     d.cache = c->d_cache;
     d.pool = c->pool;
     d.stats = c->stats;
-    d.prot = (uint32_t)prot;
+    d.prot = region_prot_flags(c, (uint32_t)prot);
     d.id = id;
     d.live = 1;
     if (cudaMemcpy(c->regions + id, &d, sizeof d, cudaMemcpyHostToDevice) != cudaSuccess)
@@ -769,6 +776,12 @@ extern "C" int ap_cache_set_policy(ap_cache_t c, int policy, uint64_t seed) {
     AP_CUDA_TRY(cudaDeviceSynchronize());
     c->h.policy = policy;
     c->h.policy_seed = seed;
+    /* the regions' drop-behind flag follows the policy */
+    for (uint32_t i = 0; i < c->reg.size(); ++i)
+        if (c->reg[i].live) {
+            const uint32_t prot = region_prot_flags(c, c->reg[i].prot);
+            AP_CUDA_TRY(cudaMemcpy(&c->regions[i].prot, &prot, 4, cudaMemcpyHostToDevice));
+        }
     return push_descriptor(c);
 }
 
@@ -844,3 +857,21 @@ extern "C" int ap_prefill(ap_cache_t c, ap_region_t r, uint64_t first, uint64_t 
     AP_CUDA_TRY(cudaGetLastError());
     return AP_OK;
 }
+
+#ifdef AP_FAULT_PROF
+/* diagnostic builds only (AP_FAULT_PROF): the fault-path phase counters */
+namespace ap {
+namespace detail {
+__device__ unsigned long long ap_fprof[16];
+}
+}  // namespace ap
+extern "C" int ap_fault_prof(uint64_t* out16, int reset) {
+    AP_CUDA_TRY(cudaDeviceSynchronize());
+    AP_CUDA_TRY(cudaMemcpyFromSymbol(out16, ap::detail::ap_fprof, 16 * sizeof(uint64_t)));
+    if (reset) {
+        static const unsigned long long zero[16] = {};
+        AP_CUDA_TRY(cudaMemcpyToSymbol(ap::detail::ap_fprof, zero, sizeof(zero)));
+    }
+    return AP_OK;
+}
+#endif

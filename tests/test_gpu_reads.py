@@ -63,6 +63,57 @@ def test_seq_copy_is_the_file(ap, dev, frames, elem, access):
         teardown(ap, cache)
 
 
+@pytest.mark.parametrize("policy", ["clock", "sequential"])
+@pytest.mark.parametrize("frames", [1, 3, 64, 4096])
+@pytest.mark.parametrize("mode", ["apointer", "raw"])
+def test_seq_queue_copy_is_the_file(ap, dev, frames, policy, mode):
+    """AP_SEQ_QUEUE (units handed out from a device counter, the C1 launch):
+    whichever warp reads a unit, every byte lands at its offset -- the file,
+    ragged tail included -- invariants hold, and 2 units per warp or fewer
+    than one unit per warp both work.  Its twin reads the zero-copy host
+    bytes through the same queue."""
+    nbytes = (1 << 20) + 3 * 4096 + 48
+    f = make_file(nbytes, seed=7)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        ap.ap_cache_set_policy(cache, ap.AP_POLICY_SEQUENTIAL if policy == "sequential"
+                               else ap.AP_POLICY_CLOCK)
+        r = ap.ap_mmap(cache, f)
+        for grid, block in ((2, 64), (148, 32), (300, 32)):
+            if frames == 1 and grid * block > 64:
+                continue
+            kw = dict(mode=ap.AP_MODE_RAW, raw_base=ap.ap_region_devptr(cache, r)) \
+                if mode == "raw" else {}
+            cfg = ap.bench_cfg(ap.AP_SEQ_QUEUE, 16, grid, block, unit_bytes=4096,
+                               out_copy=True, span_bytes=nbytes, **kw)
+            for rep in range(2):  # the counter restarts at every launch
+                out = _run(ap, cache, r, cfg, grid * block, dev, out_bytes=nbytes)
+                assert np.array_equal(out[:nbytes // 16 * 16], f[:nbytes // 16 * 16]), (grid, rep)
+        assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        teardown(ap, cache)
+
+
+def test_seq_queue_rejects_checksums_and_other_access(ap, dev):
+    """The queue's unit order is dynamic, so per-thread checksums (which
+    depend on which units a thread read) and the other access styles are
+    refused."""
+    from paper_conf_isca_shaharbs16_b200._lib import APError
+    f = make_file(1 << 20, seed=8)
+    cache = ap.ap_cache_create(64, 4096)
+    try:
+        r = ap.ap_mmap(cache, f)
+        out = torch.zeros(1 << 20, dtype=torch.uint8, device=dev)
+        for kw in (dict(out_copy=False), dict(out_copy=True, access=ap.AP_ACCESS_RANGE)):
+            cfg = ap.bench_cfg(ap.AP_SEQ_QUEUE, 16, 4, 64, unit_bytes=4096, **kw)
+            with pytest.raises(APError):
+                ap.ap_bench_read(cache, r, cfg, out)
+        ap.ap_munmap(cache, r)
+    finally:
+        teardown(ap, cache)
+
+
 @pytest.mark.parametrize("elem,unit,passes", [(16, 4096, 1), (16, 16384, 3), (4, 2048, 2),
                                               (8, 65536, 1)])
 @pytest.mark.parametrize("access", ACCESS)

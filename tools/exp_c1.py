@@ -27,8 +27,13 @@ def main():
             cache = ap.ap_cache_create(frames, 4096, 0)
             region = ap.ap_mmap(cache, f)
             ap.ap_cache_set_policy(cache, pol)
+            if os.environ.get("AP_EXP_BACKOFF"):
+                lo, hi = (int(v) for v in os.environ["AP_EXP_BACKOFF"].split(","))
+                ap.ap_cache_set_backoff(cache, lo, hi)
+            if os.environ.get("AP_EXP_SWEEP"):
+                ap.ap_cache_set_tuning(cache, 1, int(os.environ["AP_EXP_SWEEP"]), 0)
             out = torch.empty(fb, dtype=torch.uint8, device=dev)
-            bc = ap.bench_cfg(ap.AP_SEQ, 16, grid, 32, unit_bytes=4096, out_copy=True)
+            bc = ap.bench_cfg(int(os.environ.get("AP_EXP_PATTERN", ap.AP_SEQ)), 16, grid, 32, unit_bytes=4096, out_copy=True)
             ts = []
             for it in range(6):
                 ap.ap_cache_reset(cache)
