@@ -21,6 +21,8 @@ timeout 900 $N -k 'regex:^k_collage$' -s 1 -c 1 -o /tmp/ncu/r2_full_c4 -f \
   python bench.py --workload c4 --steps 1 --warmup 1 --no-cpu-baseline > gpurun_out/r2_full_c4.out 2>&1
 AP_PROF_SCHEDS=2 AP_PROF_STEPS=1 timeout 900 $N -k 'regex:^k_collage$' -s 1 -c 2 \
   -o /tmp/ncu/r2_full_c4_resident -f python tools/prof_collage.py 1048576 8 > gpurun_out/r2_full_c4_resident.out 2>&1
+timeout 900 $N -k 'regex:^k_seq_queue$' -s 1 -c 1 -o /tmp/ncu/r2_full_c1 -f \
+  python bench.py --workload c1 --steps 1 --warmup 1 --no-cpu-baseline > gpurun_out/r2_full_c1.out 2>&1
 for r in /tmp/ncu/*.ncu-rep; do
   b=$(basename $r .ncu-rep)
   python tools/ncu_summary.py $r 30 > gpurun_out/$b.txt 2>&1

@@ -193,6 +193,22 @@ for frames, policy in ((3, ap.AP_POLICY_SEQUENTIAL), (5, ap.AP_POLICY_CLOCK)):
     check(f"deref invariants frames={frames}", check_invariants(ap, c, [r], frames) == [])
     ap.ap_munmap(c, r)
     ap.ap_cache_destroy(c)
+# [r2] the C1 launch: page units from the work queue (AP_SEQ_QUEUE) under the
+# drop-behind policy (pin kept across the fault, claim-first probe), fewer
+# frames than warps
+for frames in (3, 8):
+    c = ap.ap_cache_create(frames, 4096)
+    ap.ap_cache_set_policy(c, ap.AP_POLICY_SEQUENTIAL)
+    r = ap.ap_mmap(c, fd_)
+    outq = torch.zeros(fd_.nbytes, dtype=torch.uint8, device=dev)
+    ap.ap_bench_read(c, r, ap.bench_cfg(ap.AP_SEQ_QUEUE, 16, 12, 32, unit_bytes=4096,
+                                        out_copy=True, span_bytes=fd_.nbytes), outq)
+    torch.cuda.synchronize()
+    w = fd_.nbytes // 16 * 16
+    check(f"queue frames={frames}", np.array_equal(outq.cpu().numpy()[:w], fd_[:w]))
+    check(f"queue invariants frames={frames}", check_invariants(ap, c, [r], frames) == [])
+    ap.ap_munmap(c, r)
+    ap.ap_cache_destroy(c)
 fa = make_file(1 << 21, 4)
 c = ap.ap_cache_create(4, 4096)
 r = ap.ap_mmap(c, fa)
