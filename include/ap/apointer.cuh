@@ -1093,13 +1093,25 @@ __device__ AP_SLOW_ATTR slow_out<T> deref_slow(unsigned m, uint64_t x, uint64_t 
  * caller runs the full fault path (deref_slow), which takes lanes linked
  * here as already served.  Inline and call-free, so in the common resident
  * case no register state is saved around an out-of-line call. */
-template <class T>
+template <class T, bool STREAM = false>
 __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& page,
                                            const dev_region* r, uint32_t lg,
                                            uint32_t* absent = nullptr) {
     const bool need = !(x >> 63);
     /* out-of-range / misaligned offsets: the full path reports them */
     if (__any_sync(m, need && (x + sizeof(T) > r->bytes || (x % sizeof(T)) != 0))) return false;
+    /* STREAM (the tile / range reads through relink): the pool base and the
+     * counters are read before the acquire below, which invalidates L1 --
+     * read after it, the pool base costs one more L2 round trip before the
+     * linked lanes' first loads.  The per-access miss path (inline in every
+     * dereference loop) reads them afterwards: holding them across the add
+     * there cost the loop more than the round trip (tools/exp_hit.py). */
+    const uint8_t* pool = nullptr;
+    dev_stats* rstats = nullptr;
+    if constexpr (STREAM) {
+        pool = r->pool;
+        rstats = r->stats;
+    }
     const uint64_t pg = x >> lg;
     const unsigned grp = __match_any_sync(m, need ? (((unsigned long long)r->id << 48) | pg) : ~0ull);
     const int leader = __ffs(grp) - 1;
@@ -1115,7 +1127,7 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
         /* a sequential stream (drop-behind policy) expects its next page to
          * be absent: probe with the claim (EMPTY -> LOADING, the fault
          * path's first step) and link with the add only if it is VALID */
-        const bool stream = (r->prot & REGION_DROP_BEHIND) && !r->shared;
+        const bool stream = STREAM && (r->prot & REGION_DROP_BEHIND) && !r->shared;
         if (stream) {
             old = cas_acquire(pte, PTE_EMPTY, PTE_LOADING);
             claimed = old == PTE_EMPTY;
@@ -1135,14 +1147,14 @@ __device__ __forceinline__ bool link_minor(unsigned m, uint64_t& x, uint64_t& pa
 #ifndef AP_NO_HOT_STATS /* ablation: no counters on the inline link / unlink */
     const unsigned linkedm = __ballot_sync(m, is_leader && (old >> 62) == 2);
     if (linkedm && (int)lane_id() == __ffs(m) - 1)
-        stat_add(&(r->stats + (sm_id() % STAT_SHARDS))->minor, __popc(linkedm));
+        stat_add(&((STREAM ? rstats : r->stats) + (sm_id() % STAT_SHARDS))->minor, __popc(linkedm));
 #endif
     old = __shfl_sync(m, old, leader);
     const bool ok = !need || (old >> 62) == 2;
     if (need && ok) {
         const uint64_t P = 1ull << lg;
         const uint64_t f = (old >> 32) & PTE_FRAME_MASK;
-        x = XL_VALID | ((uint64_t)(r->pool + f * P) + (x & (P - 1)));
+        x = XL_VALID | ((uint64_t)((STREAM ? pool : r->pool) + f * P) + (x & (P - 1)));
         page = pg;
     }
     /* the page was not resident (EMPTY): the fault path may claim it at once
@@ -1158,7 +1170,7 @@ __device__ __forceinline__ uint32_t absent_hint(uint32_t absent) {
 
 /* link_minor unless built with -DAP_NO_LINK_MINOR (ablation: every link
  * through the out-of-line fault path) */
-template <class T>
+template <class T, bool STREAM = false>
 __device__ __forceinline__ bool try_link_minor(unsigned m, uint64_t& x, uint64_t& page,
                                                const dev_region* r, uint32_t lg,
                                                uint32_t* absent = nullptr) {
@@ -1166,7 +1178,7 @@ __device__ __forceinline__ bool try_link_minor(unsigned m, uint64_t& x, uint64_t
     if (absent) *absent = 0;
     return false;
 #else
-    return link_minor<T>(m, x, page, r, lg, absent);
+    return link_minor<T, STREAM>(m, x, page, r, lg, absent);
 #endif
 }
 
@@ -1436,11 +1448,13 @@ struct ptr {
      * resident (link_minor), else through the fault handler. */
     __device__ __forceinline__ T deref_miss(unsigned m) {
         const uint64_t left = page;
-        const uint32_t hint = drop_stale(m, true);
+        /* (no drop-behind pin or claim-first probe here: this miss path is
+         * inline in every per-access loop, which it must not slow down; the
+         * streaming paths are the tile / range reads through relink) */
+        const uint32_t hint = drop_stale(m);
         uint32_t absent = 0;
         if (detail::try_link_minor<T>(m, x, page, r, lg, &absent)) {
             sync_fb();
-            unpin(m, hint, left);
             return detail::ld_data<T>(reinterpret_cast<const T*>(x & XL_ADDR));
         }
         const detail::slow_out<T> o =
@@ -1753,7 +1767,7 @@ struct ptr {
         AP_FP_T(tr1);
         AP_FP_ADD(m, 8, tr1 - tr0);
         uint32_t absent = 0;
-        const bool minor_ok = !__any_sync(m, !holds()) || detail::try_link_minor<T>(m, x, page, r, lg, &absent);
+        const bool minor_ok = !__any_sync(m, !holds()) || detail::try_link_minor<T, true>(m, x, page, r, lg, &absent);
         AP_FP_T(tr2);
         AP_FP_ADD(m, 9, tr2 - tr1);
         AP_FP_ADD(m, 10, 1);
