@@ -155,9 +155,15 @@ typedef struct {
                            * library is built with -DAP_COUNT_UNLINKS)           */
     uint64_t peer_fills;  /* major faults served from a peer cache (N2)           */
     uint64_t peer_bytes;  /* bytes those fills copied from peer frames            */
+    uint64_t backoff_spins;   /* = waits (SURVEY B5's name)                       */
+    uint64_t live_refcnt_sum; /* sum of the reference counts in the page tables *
+                               * now: 0 whenever no apointer is linked  */
+    int64_t err;              /* the sticky device error word (AP_OK if none),  *
+                               * read without clearing it                       */
 } ap_stats_t;
 
-/* Sum of the device counters since create/reset (synchronises the device). */
+/* Sum of the device counters since create/reset, the live reference count
+ * and the sticky error word (synchronises the device). */
 int ap_cache_stats(ap_cache_t cache, ap_stats_t* out);
 
 /* Evict every page, rebuild the free list, zero the counters: the next run

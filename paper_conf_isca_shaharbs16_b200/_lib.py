@@ -26,7 +26,8 @@ u64, u32, i32, vp, ci = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes
 class ap_stats_t(ctypes.Structure):
     _fields_ = [(n, u64) for n in ("major", "minor", "fill_bytes", "evictions", "waits",
                                    "downgrades", "nofree", "unlinks", "peer_fills",
-                                   "peer_bytes")]
+                                   "peer_bytes", "backoff_spins", "live_refcnt_sum")] + \
+               [("err", ctypes.c_int64)]
 
     def as_dict(self):
         return {n: int(getattr(self, n)) for n, _ in self._fields_}

@@ -94,6 +94,18 @@ __global__ void k_scan_pte(const uint64_t* pte, uint64_t n, int* flag) {
     if (f) atomicOr(flag, f);
 }
 
+/* sum of the reference-count fields of n entries `stride` words apart
+ * (B5's live_refcnt_sum) */
+__global__ void k_refsum(const uint64_t* pte, uint64_t n, uint64_t stride,
+                         unsigned long long* sum) {
+    unsigned long long t = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        t += pte[i * stride] & ap::PTE_RC_MASK;
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+    if ((threadIdx.x & 31) == 0 && t) atomicAdd(sum, t);
+}
+
 #ifdef AP_PT_HASH
 /* hash page table (N4 ablation): per-slot scans of one region's keys */
 __global__ void k_scan_slots(const uint64_t* slots, uint64_t n, uint64_t tag, int* flag) {
@@ -721,6 +733,26 @@ extern "C" int ap_cache_stats(ap_cache_t c, ap_stats_t* out) {
         t.peer_fills += x.peer_fills;
         t.peer_bytes += x.peer_bytes;
     }
+    t.backoff_spins = t.waits;
+    /* live references: the count fields of every page-table entry */
+    unsigned long long* d_sum = nullptr;
+    AP_CUDA_TRY(cudaMalloc(&d_sum, sizeof(unsigned long long)));
+    cudaError_t e = cudaMemset(d_sum, 0, sizeof(unsigned long long));
+#ifdef AP_PT_HASH
+    if (e == cudaSuccess) k_refsum<<<c->num_sms * 4, 256>>>(c->slots + 1, 1ull << c->slot_bits, 2, d_sum);
+#else
+    for (auto& rg : c->reg)
+        if (e == cudaSuccess && rg.live) k_refsum<<<c->num_sms * 4, 256>>>(rg.pte, rg.npages, 1, d_sum);
+#endif
+    if (e == cudaSuccess) e = cudaGetLastError();
+    unsigned long long sum = 0;
+    if (e == cudaSuccess) e = cudaMemcpy(&sum, d_sum, sizeof sum, cudaMemcpyDeviceToHost);
+    cudaFree(d_sum);
+    AP_CUDA_TRY(e);
+    t.live_refcnt_sum = sum;
+    int err = 0; /* the sticky error word, not cleared (ap_last_device_error clears it) */
+    AP_CUDA_TRY(cudaMemcpy(&err, c->err, sizeof(int), cudaMemcpyDeviceToHost));
+    t.err = err;
     *out = t;
     return AP_OK;
 }

@@ -95,6 +95,34 @@ def test_seq_queue_copy_is_the_file(ap, dev, frames, policy, mode):
         teardown(ap, cache)
 
 
+def test_stats_live_refcnt_sum_and_err(ap, dev):
+    """SURVEY B5's counters: live_refcnt_sum is the page tables' reference
+    counts (0 once every apointer is gone; equal to the sum over
+    the PTE dump), backoff_spins = waits, err = the sticky error word (read
+    without clearing it)."""
+    nbytes = (1 << 21) + 4096 + 48
+    f = make_file(nbytes, seed=9)
+    cache = ap.ap_cache_create(8, 4096)
+    try:
+        r = ap.ap_mmap(cache, f)
+        cfgs = [ap.bench_cfg(ap.AP_SEQ_QUEUE, 16, 20, 32, unit_bytes=4096, out_copy=True,
+                             span_bytes=nbytes),
+                ap.bench_cfg(ap.AP_UNIFORM, 4, 6, 128, reads_per_thread=5, seed=3),
+                ap.bench_cfg(ap.AP_DIVERGENT, 4, 4, 64, reads_per_thread=3, page_bytes=4096,
+                             seed=5)]
+        for cfg in cfgs:
+            out = torch.zeros(max(nbytes, 20 * 32 * 8), dtype=torch.uint8, device=dev)
+            ap.ap_bench_read(cache, r, cfg, out)
+            st = ap.ap_cache_stats(cache)
+            rc = (ap.ap_region_dump_pte(cache, r) & np.uint64(0xffffffff)).sum()
+            assert st["live_refcnt_sum"] == int(rc) == 0
+            assert st["err"] == 0 and st["backoff_spins"] == st["waits"]
+            assert ap.ap_last_device_error(cache) == 0
+        ap.ap_munmap(cache, r)
+    finally:
+        teardown(ap, cache)
+
+
 def test_seq_queue_rejects_checksums_and_other_access(ap, dev):
     """The queue's unit order is dynamic, so per-thread checksums (which
     depend on which units a thread read) and the other access styles are
