@@ -600,6 +600,8 @@ def main():
                         "(CUDA IPC + system-scope atomics, no collective) or one NCCL "
                         "gather / MIN reduce after the kernel")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-reads", action="store_true",
+                   help="default workload only: skip the embedded C1 / C3 objects")
     p.add_argument("--no-collage", action="store_true",
                    help="default workload only: skip the embedded C4 collage object")
     args = p.parse_args()
@@ -646,6 +648,18 @@ def main():
         cres = bench_collage.run_collage(cargs, torch, dev, rank, world, dist, timed, ClockSampler,
                                          host_link_peak, light=True)
         coll_all = gather_all(cres, ("got", "is_copy", "src"), rank, world, dist)
+    reads_all = {}
+    if args.workload == "c2" and not args.no_reads:
+        # C1 and C3 (BASELINE.json configs[0], [2]: the paper's page-fault
+        # microbenchmark regimes) ride along as well
+        import copy
+        import bench_reads
+        for w in ("c1", "c3"):
+            rargs = copy.copy(args)
+            rargs.workload, rargs.policy = w, None
+            rres = bench_reads.run_reads(rargs, torch, dev, rank, world, dist, timed, ClockSampler,
+                                         host_link_peak, aligned_empty)
+            reads_all[w] = (rargs, gather_all(rres, (), rank, world, dist))
     res_all = gather_all(res, drop, rank, world, dist)
     if rank == 0:
         if args.workload in ("c4", "c5"):
@@ -660,6 +674,9 @@ def main():
                 cargs = copy.copy(args)
                 cargs.workload = "c4"
                 line["collage_c4"] = bench_collage.collage_summary(cargs, coll_all, world)
+            for w, (rargs, rall) in reads_all.items():
+                import bench_reads
+                line[f"reads_{w}"] = bench_reads.reads_summary(rargs, rall, world, METRIC)
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()

@@ -182,3 +182,20 @@ def emit_reads(args, res_all, world, METRIC):
                                 "cores": r0["parity"]["cores"], "kind": "oracle",
                                 "sample": "the whole read set, plain file indexing; bytes read / s"}
     return line
+
+
+def reads_summary(args, res_all, world, METRIC):
+    """The C1 / C3 line (emit_reads) as a sub-object of the default line: the
+    driver then runs these configs too (cold cache per step, device-timed,
+    parity vs the oracle on rank 0)."""
+    line = emit_reads(args, res_all, world, METRIC)
+    times = [t for r in res_all for t in r["times"]]
+    mean = sum(times) / len(times)
+    std = (sum((t - mean) ** 2 for t in times) / max(len(times) - 1, 1)) ** 0.5
+    keep = ("value", "unit", "ms_per_step", "dtype", "config", "fault_bound", "roofline",
+            "parity_vs_oracle", "cpu_baseline", "clocks")
+    out = {k: line[k] for k in keep if k in line}
+    out["value_note"] = "page-fill bytes per second over the host link (the fault path's rate)"
+    out["step_times"] = {"mean_ms": round(mean * 1e3, 4), "std_ms": round(std * 1e3, 4),
+                         "n": len(times)}
+    return out
