@@ -600,6 +600,8 @@ def main():
                         "(CUDA IPC + system-scope atomics, no collective) or one NCCL "
                         "gather / MIN reduce after the kernel")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-c5", action="store_true",
+                   help="default workload only: skip the embedded C5 collage object (40 GB host file)")
     p.add_argument("--no-reads", action="store_true",
                    help="default workload only: skip the embedded C1 / C3 objects")
     p.add_argument("--no-collage", action="store_true",
@@ -648,6 +650,19 @@ def main():
         cres = bench_collage.run_collage(cargs, torch, dev, rank, world, dist, timed, ClockSampler,
                                          host_link_peak, light=True)
         coll_all = gather_all(cres, ("got", "is_copy", "src"), rank, world, dist)
+        del cres
+    c5_all = None
+    if args.workload == "c2" and not args.no_collage and not args.no_c5:
+        # and C5 (configs[4]: 10M records, 40 GB pinned file, the multi-GPU
+        # collage; one step per timed step at this --gpus N)
+        import copy
+        import bench_collage
+        c5args = copy.copy(args)
+        c5args.workload, c5args.stride = "c5", 4096
+        c5res = bench_collage.run_collage(c5args, torch, dev, rank, world, dist, timed, ClockSampler,
+                                          host_link_peak, light=True)
+        c5_all = gather_all(c5res, ("got", "is_copy", "src"), rank, world, dist)
+        del c5res
     reads_all = {}
     if args.workload == "c2" and not args.no_reads:
         # C1 and C3 (BASELINE.json configs[0], [2]: the paper's page-fault
@@ -674,6 +689,12 @@ def main():
                 cargs = copy.copy(args)
                 cargs.workload = "c4"
                 line["collage_c4"] = bench_collage.collage_summary(cargs, coll_all, world)
+            if c5_all is not None:
+                import copy
+                import bench_collage
+                c5args = copy.copy(args)
+                c5args.workload = "c5"
+                line["collage_c5"] = bench_collage.collage_summary(c5args, c5_all, world)
             for w, (rargs, rall) in reads_all.items():
                 import bench_reads
                 line[f"reads_{w}"] = bench_reads.reads_summary(rargs, rall, world, METRIC)

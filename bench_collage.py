@@ -504,6 +504,8 @@ def collage_summary(args, res_all, world):
         "fill_frac_of_host_link": round(st["fill_bytes"] / float(np.mean(r0["times"])) / 1e9 /
                                         r0["link"], 4),
         "e2e_s": round(max(float(np.mean(r["e2e"])) for r in res_all), 6),
+        "setup_s": {"generate": round(r0["t_gen"], 2), "pin": round(r0["t_pin"], 2),
+                    "index": round(r0["t_index"], 3)},
     }
     raw = r0.get("raw")
     if raw:
