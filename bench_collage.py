@@ -45,8 +45,10 @@ def _collage_config(name):
     return dict(name="c5", N=10_000_000, W=8192, H=8192, L=4, K=8, bb=16, w=40000,
                 frames=524288, page=4096, stride=4096,
                 workload="C5: 10M tiles in a 40.96 GB pinned host file, 8192x8192 target, LSH "
-                         "L=4 K=8 2^16 buckets, query blocks partitioned over the ranks, 2 GiB "
-                         "page cache per GPU (cold per step), one NCCL gather of the winners")
+                         "L=4 K=8 2^16 buckets, work partitioned over the ranks (--partition), 2 "
+                         "GiB page cache per GPU (cold per step); N > 1: winners folded into rank "
+                         "0's array by the kernels (--combine fused) or one NCCL gather / MIN "
+                         "reduce (--combine nccl)")
 
 
 def numa_interleave(arr):
