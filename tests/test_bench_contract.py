@@ -8,6 +8,8 @@ import sys
 
 import pytest
 
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
@@ -42,3 +44,30 @@ def test_our_arm_fails_loudly_without_a_gpu():
                        capture_output=True, text=True, timeout=600)
     assert r.returncode != 0
     assert not [ln for ln in r.stdout.splitlines() if ln.strip().startswith("{")]
+
+
+def _fake_reads_res(times, name="c1"):
+    import bench_reads
+    cfg = bench_reads.read_config(name, 8)
+    cfg["policy"] = "sequential"
+    st = dict(fill_bytes=16 << 20, major=4096, minor=0, evictions=4032, waits=10,
+              downgrades=0, nofree=10)
+    return dict(cfg=cfg, times=times, stats=[st] * len(times), err=0, link=55.0, raw_t=3e-4,
+                raw_equal=True, reads=(16 << 20) // 16, clocks={}, parity=None,
+                other_policies={})
+
+
+def test_reads_summary_takes_the_slowest_rank():
+    """The C1 / C3 objects of the default line: value = the whole job's fill
+    bytes over the slowest rank's mean step (the contract's max over ranks)."""
+    import argparse
+    import bench_reads
+    sys.path.insert(0, ROOT)
+    args = argparse.Namespace(steps=2, warmup=3, workload="c1")
+    fast, slow = _fake_reads_res([1e-3, 1e-3]), _fake_reads_res([2e-3, 2e-3])
+    out = bench_reads.reads_summary(args, [fast, slow], 2, "m")
+    assert out["ms_per_step"] == 2.0
+    assert out["value"] == round(2 * (16 << 20) / 2e-3 / 1e9, 3)
+    assert out["step_times"]["n"] == 4 and out["step_times"]["mean_ms"] == 1.5
+    assert out["roofline"]["bound"] == "host_link" and 0 < out["roofline"]["frac"]
+    assert "parity_vs_oracle" not in out  # rank 0 ran no oracle here
