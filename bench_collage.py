@@ -509,6 +509,17 @@ def collage_summary(args, res_all, world):
         "setup_s": {"generate": round(r0["t_gen"], 2), "pin": round(r0["t_pin"], 2),
                     "index": round(r0["t_index"], 3)},
     }
+    # the collage kernel is fill-bound: its roofline is the host link (page
+    # fill bytes per second of the device-timed step, one launch per step)
+    fill_rate = st["fill_bytes"] / float(np.mean(r0["times"])) / 1e9
+    from bench import ncu_traffic
+    out["roofline"] = {"bound": "host_link", "achieved": round(fill_rate, 3),
+                       "peak": round(r0["link"], 3), "unit": "GB/s",
+                       "frac": round(fill_rate / r0["link"], 4),
+                       "traffic": ncu_traffic("k_collage<8, apointer>") if cfg["name"] == "c4" else None,
+                       "algorithmic_bytes_per_launch": int(st["fill_bytes"]),
+                       "kernel": "k_collage<8, apointer> (the step's record-id windows fused in one launch)",
+                       "peak_source": "host->device cudaMemcpy from pinned memory, this run"}
     raw = r0.get("raw")
     if raw:
         bound = raw["distinct_pages"] * cfg["page"] / (r0["link"] * 1e9)
@@ -525,6 +536,9 @@ def collage_summary(args, res_all, world):
         full_blocks = r0["b1"] - r0["b0"]
         out["oracle_s"] = round(p["cpu_s"] * full_blocks / p["blocks"], 4)
         out["oracle_cores"] = p["cores"]
+        if p["blocks"] < full_blocks:
+            out["oracle_s_note"] = (f"the oracle ran {p['blocks']} of {full_blocks} blocks; "
+                                    "oracle_s scales its time to all blocks")
     if r0.get("gathered_parity"):
         out["gathered_parity_vs_oracle"] = r0["gathered_parity"]
     return out
