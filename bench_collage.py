@@ -166,7 +166,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     tgt_host = torch.from_numpy(img).pin_memory()
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
-    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 12, "c5": 12}.get(cfg["name"], 0)
+    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 32, "c5": 12}.get(cfg["name"], 0)
     id_chunks = id_chunks if args.schedule in (2, 3) else 0
     if i1:  # the windows split this rank's record slice
         id_chunks = max(1, -(-id_chunks // world))
@@ -257,7 +257,8 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         inp_raw = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                                         cfg["N"], cfg["stride"], group=args.group, block_begin=b0,
                                 block_count=b1 - b0, mode=ap.AP_MODE_RAW, raw_base=dcopy,
-                                schedule=args.schedule)
+                                schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0,
+                                id_begin=i0, id_end=i1)  # this rank's share, like inp
         win_raw = torch.empty_like(win)
         for _ in range(2):
             timed(torch, lambda: ap.ap_collage_run(cache, region, inp_raw, win_raw, stream), stream)
@@ -288,11 +289,13 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
         for g in (1, 2, 4, 8):
             inp_g = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                                   cfg["N"], cfg["stride"], group=g, block_begin=b0,
-                                  block_count=b1 - b0, schedule=args.schedule)
+                                  block_count=b1 - b0, schedule=args.schedule, unit_begin=u0,
+                                  unit_count=u1 - u0, id_begin=i0, id_end=i1)
             inp_gr = ap.collage_in(tgt, cfg["W"], cfg["H"], pd, bd, cfg["w"], cfg["bb"], off, ids,
                                    cfg["N"], cfg["stride"], group=g, block_begin=b0,
                                    block_count=b1 - b0, mode=ap.AP_MODE_RAW, raw_base=dcopy,
-                                   schedule=args.schedule)
+                                   schedule=args.schedule, unit_begin=u0, unit_count=u1 - u0,
+                                   id_begin=i0, id_end=i1)
             wg, wr = torch.empty_like(win), torch.empty_like(win)
             for _ in range(2):
                 ap.ap_collage_run(big, rb, inp_g, wg, stream)
