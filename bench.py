@@ -589,8 +589,9 @@ def main():
                         "caches one shard of the file), the sorted units, or the image")
     p.add_argument("--id-chunks", type=int, default=None,
                    help="collage record-id windows (ap_collage_in.id_chunks; 0 = off; "
-                        "default 12 for c4 and c5 (measured: C4 8/12/16 -> 30.3/29.2/29.1 ms, "
-                        "C5 8/12/16/24 -> 0.608/0.594/0.598/0.648 s)")
+                        "default 32 for c4, 96 for c5 (fused windows; measured C4 12/32/64 -> "
+                        "28.1/27.1/27.1 ms, C5 12/24/48/96 -> 0.589/0.541/0.495/0.486 s, "
+                        "profiles/r02_collage_warp_units.txt)")
     p.add_argument("--reads", type=int, default=8, help="reads per thread (C2)")
     p.add_argument("--policy", default=None, choices=["clock", "sequential"],
                    help="c1/c3 eviction policy (default: sequential drop-behind for the "

@@ -166,7 +166,7 @@ def run_collage(args, torch, dev, rank, world, dist, timed, ClockSampler, host_l
     tgt_host = torch.from_numpy(img).pin_memory()
     tgt = tgt_host.to(dev)
     win = torch.empty((b1 - b0, 2), dtype=torch.int32, device=dev)
-    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 32, "c5": 12}.get(cfg["name"], 0)
+    id_chunks = args.id_chunks if args.id_chunks is not None else {"c4": 32, "c5": 96}.get(cfg["name"], 0)
     id_chunks = id_chunks if args.schedule in (2, 3) else 0
     if i1:  # the windows split this rank's record slice
         id_chunks = max(1, -(-id_chunks // world))

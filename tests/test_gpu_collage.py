@@ -336,3 +336,40 @@ def test_empty_candidate_sets_give_the_sentinel(ap, group, schedule):
         ap.ap_munmap(cache, r)
     finally:
         teardown(ap, cache)
+
+
+@pytest.mark.parametrize("group", [4, 8])
+@pytest.mark.parametrize("stride,frames", [(4096, 64), (4096, 5000), (3072, 40)])
+def test_collage_warp_items_many_windows(ap, group, stride, frames):
+    """A step with >= 2^20 (window, unit) items runs one warp per item
+    (k_collage_wunit, with the precomputed window bounds and the empty-window
+    exit): 1024 blocks x 4 tables x 256 windows.  Winners equal the one-pass
+    run and the oracle (on its own index), with a cache smaller and larger
+    than the touched records and with records straddling pages."""
+    dev = torch.device("cuda:0")
+    n, w, bb, L, K = 4096, 2500, 8, 4, 5
+    W, H = 1024, 1024
+    recs, proj, bias, img, *_ = _setup(n, W, H, L, K, w, bb, seed=12, stride=stride)
+    cache = ap.ap_cache_create(frames, 4096)
+    try:
+        r = ap.ap_mmap(cache, recs)
+        off, ids, pd, bd = _gpu_index(ap, cache, r, n, stride, proj, bias, w, bb, dev)
+        tgt = torch.from_numpy(img).to(dev)
+        nb = (W // 32) * (H // 32)
+        one = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride,
+                                                  group=group, schedule=2), one)
+        win = torch.zeros((nb, 2), dtype=torch.int32, device=dev)
+        ap.ap_cache_reset(cache)
+        ap.ap_collage_run(cache, r, ap.collage_in(tgt, W, H, pd, bd, w, bb, off, ids, n, stride,
+                                                  group=group, schedule=2, id_chunks=256), win)
+        torch.cuda.synchronize()
+        assert ap.ap_last_device_error(cache) == 0
+        assert torch.equal(win, one)
+        o_off, o_ids = oracle.build_index(recs, stride, n, proj, bias, w, bb)
+        want = oracle.collage(img, proj, bias, w, bb, recs, stride, n, o_off, o_ids)
+        assert np.array_equal(win.cpu().numpy().view(np.uint32), want)
+        assert check_invariants(ap, cache, [r], frames) == []
+        ap.ap_munmap(cache, r)
+    finally:
+        teardown(ap, cache)
