@@ -402,6 +402,9 @@ def emit_collage(args, res_all, world, METRIC):
     st = r0["stats"][-1]
     fill = st["fill_bytes"]
     t0 = sum(r0["times"]) / args.steps
+    # C5's (window, unit) items run one per warp (k_collage_wunit, >= 2^20 items)
+    kname = (f"k_collage_wunit<{args.group}, apointer>" if cfg["name"] == "c5"
+             else f"k_collage<{args.group}, apointer>")
     line = {
         "metric": METRIC, "value": round(tmax, 6), "unit": "s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tmax * 1e3, 3),
@@ -440,13 +443,12 @@ def emit_collage(args, res_all, world, METRIC):
         "roofline": {"bound": "host_link", "achieved": round(fill / t0 / 1e9, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
                      "frac": round(fill / t0 / 1e9 / r0["link"], 4),
-                     "traffic": (lambda tr: None if tr is None else tr * max(1, r0["id_chunks"]))(
-                         _traffic(f"k_collage<{args.group}, apointer>")),
-                     "traffic_note": "DRAM bytes per step = the ncu --set full capture of one "
-                                     "k_collage launch (one record-id window pass) x the "
-                                     "step's id_chunks launches",
+                     "traffic": _traffic(kname),
+                     "traffic_note": "DRAM bytes of one step = one launch (the record-id windows "
+                                     "are fused), from the committed ncu --set full capture "
+                                     "(profiles/traffic.json)",
                      "algorithmic_bytes_per_step": int(fill),
-                     "kernel": f"k_collage<{args.group}, apointer>",
+                     "kernel": kname,
                      "peak_source": "host->device cudaMemcpy from pinned memory, this run"},
         "e2e": {"value": round(max(np.mean(r["e2e"]) for r in res_all), 6), "unit": "s",
                 "h2d_bytes_per_step": r0["h2d"], "d2h_bytes_per_step": r0["d2h"],
@@ -515,13 +517,22 @@ def collage_summary(args, res_all, world):
     # the collage kernel is fill-bound: its roofline is the host link (page
     # fill bytes per second of the device-timed step, one launch per step)
     fill_rate = st["fill_bytes"] / float(np.mean(r0["times"])) / 1e9
+    # C5's 25 M (window, unit) items run one per warp (k_collage_wunit)
+    kname = "k_collage_wunit<8, apointer>" if cfg["name"] == "c5" else "k_collage<8, apointer>"
+    if cfg["name"] == "c5":
+        out["traffic_note"] = ("ncu DRAM bytes per launch (profiles/r02_full_c5.txt): 87 GB of reads are "
+                               "the candidates' payload re-read from the frames (~120 GB of record "
+                               "reads, L2 serves the rest) and 51 GB of writes = 24 GB of fills + the "
+                               "rest, L2 evictions of local-memory (spill) lines of the fault path "
+                               "(8.2 G local store sectors per launch, 3.6 G of them L1 misses); HBM "
+                               "runs at 0.28 TB/s, the host link is the bound")
     from bench import ncu_traffic
     out["roofline"] = {"bound": "host_link", "achieved": round(fill_rate, 3),
                        "peak": round(r0["link"], 3), "unit": "GB/s",
                        "frac": round(fill_rate / r0["link"], 4),
-                       "traffic": ncu_traffic("k_collage<8, apointer>") if cfg["name"] == "c4" else None,
+                       "traffic": ncu_traffic(kname),
                        "algorithmic_bytes_per_launch": int(st["fill_bytes"]),
-                       "kernel": "k_collage<8, apointer> (the step's record-id windows fused in one launch)",
+                       "kernel": kname + " (the step's record-id windows fused in one launch)",
                        "peak_source": "host->device cudaMemcpy from pinned memory, this run"}
     raw = r0.get("raw")
     if raw:
