@@ -280,6 +280,13 @@ extern "C" int ap_cache_create(uint64_t frames, uint32_t page_size, int device, 
     c->h.nfree = frames;
     c->h.policy_seed = 0;
     c->h.timeout_ns = 20000ull * 1000000ull;
+    /* AP_TIMEOUT_MS (environment, diagnostics): a shorter fault-path
+     * watchdog for every cache of the process, so a wait that cannot end
+     * reports ERR_TIMEDOUT in seconds instead of tens of seconds */
+    if (const char* e = getenv("AP_TIMEOUT_MS")) {
+        const unsigned long long ms = strtoull(e, nullptr, 10);
+        if (ms) c->h.timeout_ns = ms * 1000000ull;
+    }
     c->h.log2_page = c->log2_page;
     c->h.policy = ap::POLICY_CLOCK;
     c->h.max_claims = 1;
