@@ -188,7 +188,9 @@ int ap_cache_set_policy(ap_cache_t cache, int policy, uint64_t seed);
 /* Fault-path tunables: max_claims = pages one warp claims per fault round
  * (1 = the paper's sequential handling); sweep_steps = clock
  * steps (32 frames each) before an allocation gives up and backs off;
- * timeout_ms = watchdog for one dereference (0 = default 20000). */
+ * timeout_ms = watchdog for one dereference (0 = default 20000; a new cache
+ * takes its default from the environment variable AP_TIMEOUT_MS if set, a
+ * diagnostics aid). */
 int ap_cache_set_tuning(ap_cache_t cache, uint32_t max_claims, uint32_t sweep_steps,
                         uint32_t timeout_ms);
 
