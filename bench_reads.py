@@ -136,6 +136,18 @@ def run_reads(args, torch, dev, rank, world, dist, timed, ClockSampler, host_lin
                 other_policies=other)
 
 
+def _traffic(kernel):
+    """DRAM bytes per launch of `kernel` from the committed ncu capture
+    (profiles/traffic.json), or None."""
+    import json
+    try:
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles",
+                               "traffic.json")) as f:
+            return json.load(f)[kernel]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
 def emit_reads(args, res_all, world, METRIC):
     r0 = res_all[0]
     cfg = r0["cfg"]
@@ -170,7 +182,11 @@ def emit_reads(args, res_all, world, METRIC):
                                            for k, v in r0.get("other_policies", {}).items()}},
         "roofline": {"bound": "host_link", "achieved": round(st["fill_bytes"] / t0 / 1e9, 3),
                      "peak": round(r0["link"], 3), "unit": "GB/s",
-                     "frac": round(st["fill_bytes"] / t0 / 1e9 / r0["link"], 4), "traffic": None,
+                     "frac": round(st["fill_bytes"] / t0 / 1e9 / r0["link"], 4),
+                     "traffic": _traffic("k_seq_queue<uint4, apointer>" if cfg["name"] == "c1"
+                                         else "k_random<uint32_t, DIVERGENT, apointer>"),
+                     "kernel": ("k_seq_queue<uint4, apointer>" if cfg["name"] == "c1"
+                                else "k_random<uint32_t, DIVERGENT, apointer>"),
                      "algorithmic_bytes_per_launch": int(st["fill_bytes"]),
                      "peak_source": "host->device cudaMemcpy from pinned memory, this run"},
         "gpu_launches": args.steps, "clocks": r0["clocks"],

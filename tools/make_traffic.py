@@ -34,6 +34,8 @@ tj = {
     "k_random<uint32_t, UNIFORM, apointer> resident (M2r)": entry(f"profiles/{R}_full_k_random.txt", 0, "M2r: uniform 4-B reads over the resident GiB"),
     "k_random<uint32_t, UNIFORM, raw> resident (M2r)": entry(f"profiles/{R}_full_k_random.txt", 1, "the raw gather twin"),
     "k_collage<8, apointer>": entry(f"profiles/{R}_full_c4.txt", 0, "one launch = a whole cold C4 step (the 12 record-id window passes fused into one launch)"),
+    "k_seq_queue<uint4, apointer>": entry(f"profiles/{R}_full_c1.txt", 0, "one C1 step: the 16 MiB file and its 64 frames live in L2, so DRAM sees almost nothing"),
+    "k_random<uint32_t, DIVERGENT, apointer>": entry(f"profiles/{R}_full_c3.txt", 0, "one C3 step, cold 256 MiB cache: fills recycle frames whose dirty lines L2 absorbs, so DRAM writes are below the fill bytes"),
     "k_collage_wunit<8, apointer>": entry(f"profiles/{R}_full_c5.txt", 0, "one launch = a whole cold C5 step (96 record-id windows, one warp per (window, unit) item)"),
     "k_collage<8, apointer> resident": entry(f"profiles/{R}_full_c4_resident.txt", 0, "cache holds every record"),
     "k_collage<8, raw> resident": entry(f"profiles/{R}_full_c4_resident.txt", 1, "raw twin on an HBM copy"),
