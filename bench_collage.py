@@ -90,6 +90,12 @@ def _shm_records(cfg, rank, world, dist):
     nbytes = cfg["N"] * cfg["stride"]
     path = f"/dev/shm/apb_{cfg['name']}_{cfg['N']}_{cfg['stride']}_{DS_SEED}.bin"
     done = path + ".ok"
+    if rank == 0 and os.environ.get("AP_REUSE_SHM") != "1":
+        # a file left by an earlier process is not reused (a timing must not
+        # depend on what ran before on the box); AP_REUSE_SHM=1 keeps it
+        for f_ in (done, path):
+            if os.path.exists(f_):
+                os.remove(f_)
     if rank == 0 and not os.path.exists(done):
         with open(path, "wb") as fh:
             fh.truncate(nbytes)
