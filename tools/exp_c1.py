@@ -17,7 +17,7 @@ def aligned_empty(n, align=4096):
 def main():
     dev = torch.device("cuda:0")
     stream = torch.cuda.current_stream()
-    fb = 16 << 20
+    fb = int(os.environ.get("AP_EXP_FILE_MB", 16)) << 20
     f = synth.fill_file(aligned_empty(fb), 1)
     pol = int(os.environ.get("AP_EXP_POLICY", ap.AP_POLICY_SEQUENTIAL))
     fl = [int(v) for v in os.environ.get("AP_EXP_FRAMES", "64,96,128,148,192,256,512,4096").split(",")]
