@@ -46,10 +46,45 @@ def env_rank():
             int(os.environ.get("WORLD_SIZE", 1)))
 
 
+# NUMA node of this rank's GPU (main() puts it in AP_BENCH_NODE): host
+# "files" the bench creates are bound to it before their first touch, so the
+# fault path's zero-copy fills read the socket the GPU's PCIe link hangs off
+# (AP_NUMA_LOCAL=0: off)
+
+
+def gpu_numa_node(torch, dev):
+    """The host NUMA node of `dev` from sysfs (None if unknown)."""
+    try:
+        pr = torch.cuda.get_device_properties(dev)
+        bus = f"{pr.pci_domain_id:04x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+        with open(f"/sys/bus/pci/devices/{bus}/numa_node") as f:
+            n = int(f.read().strip())
+        return n if n >= 0 else None
+    except Exception:
+        return None
+
+
+def numa_bind(arr, node):
+    """mbind(MPOL_BIND) the pages of a not-yet-touched host buffer to `node`."""
+    import ctypes
+    libc = ctypes.CDLL(None, use_errno=True)
+    page = 4096
+    addr = arr.ctypes.data & ~(page - 1)
+    length = arr.ctypes.data + arr.nbytes - addr
+    nm = ctypes.c_ulong(1 << node)
+    SYS_mbind, MPOL_BIND = 237, 2  # x86_64
+    return libc.syscall(SYS_mbind, ctypes.c_void_p(addr), ctypes.c_ulong(length), MPOL_BIND,
+                        ctypes.byref(nm), ctypes.c_ulong(node + 2), 0) == 0
+
+
 def aligned_empty(nbytes, align=1 << 21):
     raw = np.empty(nbytes + align, dtype=np.uint8)
     off = (-raw.ctypes.data) % align
-    return raw[off:off + nbytes]
+    arr = raw[off:off + nbytes]
+    node = os.environ.get("AP_BENCH_NODE")  # set by main() (other modules import bench anew)
+    if node:
+        numa_bind(arr, int(node))
+    return arr
 
 
 def ncu_traffic(kernel):
@@ -620,6 +655,10 @@ def main():
     local_dev = 0 if share else local
     torch.cuda.set_device(local_dev)
     dev = torch.device("cuda", local_dev)
+    if os.environ.get("AP_NUMA_LOCAL", "1") == "1":
+        node = gpu_numa_node(torch, dev)
+        if node is not None:
+            os.environ["AP_BENCH_NODE"] = str(node)
     dist = None
     if world > 1:
         import torch.distributed as dist
