@@ -12,7 +12,9 @@ from helpers import check_invariants, make_file, teardown
 
 pytestmark = pytest.mark.gpu
 
-CASES = list(range(24))
+# AP_STRESS_CASES="a-b" (a soak run): seeds a .. b-1 instead of the 24 default
+_rng = __import__("os").environ.get("AP_STRESS_CASES")
+CASES = list(range(*map(int, _rng.split("-")))) if _rng else list(range(24))
 
 
 def _cfg(seed):
