@@ -410,10 +410,21 @@ __device__ __forceinline__ uint64_t* pt_must(const dev_region* r, uint64_t pg) {
 #else
 #define AP_PTE_AT(r, pg) ::ap::detail::pt_find((r), (pg), false)
 #endif
-/* the probe is a leader-only loop of data-dependent length: reconverge the
- * warp after it, so later __activemask()-based operations see every lane */
+/* The probe is a leader-only loop of data-dependent length.  The warp is NOT
+ * reconverged with __syncwarp(m) after it: at some call sites m was taken
+ * before the warp diverged, and the barrier then waited forever for lanes
+ * parked at another one -- the hash build's round-2 hang (random collage
+ * case 8 hung in 8 of 8 runs with the barrier, passed 8 of 8 without).  The
+ * _sync intrinsics that follow synchronise their own masks; a later
+ * __activemask() may see a subset of the lanes, which only splits the
+ * warp-aggregated links and unlinks into smaller groups.
+ * -DAP_PT_RECONVERGE_SYNC restores the barrier (diagnostic). */
 #define AP_PTE_FIND(r, pg) ::ap::detail::pt_find((r), (pg), false) /* may miss */
+#ifdef AP_PT_RECONVERGE_SYNC
 #define AP_PT_RECONVERGE(m) __syncwarp(m)
+#else
+#define AP_PT_RECONVERGE(m) ((void)0)
+#endif
 #else
 #define AP_PTE_FIND(r, pg) ((r)->pte + (pg))
 #define AP_PT_RECONVERGE(m) ((void)0)

@@ -11,9 +11,9 @@ import sys
 
 import pytest
 
-# Opt-in (AP_RUN_PT_HASH=1): the hash build can still hang a fault-path wait
-# until the 20 s watchdog under concurrent eviction, so the default -m gpu
-# run does not include it.
+# Opt-in (AP_RUN_PT_HASH=1): the hash build still leaks a reference count
+# now and then under concurrent eviction (its round-2 hang is fixed), so the
+# default -m gpu run does not include it.
 pytestmark = [pytest.mark.gpu,
               pytest.mark.skipif(not os.environ.get("AP_RUN_PT_HASH"),
                                  reason="N4 hash-table ablation: opt-in, AP_RUN_PT_HASH=1")]
@@ -22,9 +22,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 LIB = os.path.join(ROOT, "paper_conf_isca_shaharbs16_b200", "libapointer_hash.so")
 
 
-@pytest.mark.xfail(reason="open: under concurrent eviction the hash build occasionally leaks a "
-                          "reference count or faults on a stale frame (the dense build, the "
-                          "product, is clean); see DESIGN.md §10", strict=False)
+@pytest.mark.xfail(reason="open: the hash build passes the suites in most runs but now and "
+                          "then leaks a reference count under concurrent eviction (e.g. "
+                          "test_sequential_policy_drop_behind[uniform-64]) and faults at the C2 "
+                          "bench scale; the dense build, the product, is clean; DESIGN.md §10",
+                   strict=False)
 def test_hash_page_table_passes_the_parity_suites():
     assert os.path.exists(LIB), "build libapointer_hash.so (make)"
     env = dict(os.environ, AP_LIB_PATH=LIB)
@@ -33,7 +35,8 @@ def test_hash_page_table_passes_the_parity_suites():
                            cwd=ROOT, env=env, capture_output=True, text=True, timeout=300)
     assert "hash-table page table" in probe.stdout, probe.stdout + probe.stderr
     r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
-                        "tests/test_gpu_reads.py", "tests/test_gpu_collage.py"],
+                        "tests/test_gpu_reads.py", "tests/test_gpu_collage.py",
+                        "tests/test_gpu_collage_stress.py"],
                        cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-4000:] + r.stderr[-2000:]
     assert " passed" in r.stdout
